@@ -1,0 +1,137 @@
+"""Pins for the RS oracle (SURVEY.md 8(c) PIN-9, PIN-10, PIN-12 and special
+cases that reduce to closed forms or to scipy's Faddeeva function)."""
+from fractions import Fraction
+
+import numpy as np
+import pytest
+from scipy.special import wofz
+
+import gtr_inputs.rs as RS
+import gtr_inputs.xs as X
+
+A_LCG = 2806196910506780709
+M = 1 << 63
+
+
+def step(s):
+    return (A_LCG * s + 1) % M
+
+
+def energies(seed, n):
+    out, s = [], seed
+    for _ in range(n):
+        out.append(float(Fraction(step(s), M)))
+        s = step(step(s))
+    return out
+
+
+# ---------------------------------------------------------------- PIN-9
+def test_faddeeva_inner_region_vs_scipy(orc):
+    # Abrarov N=10, Tm=12 series: accurate to ~1e-3 relative in the upper
+    # half plane for |z| < 6 (measured bound 9.1e-4 on this grid).
+    for x in np.linspace(-5.5, 5.5, 45):
+        for y in (0.05, 0.3, 1.0, 2.5, 4.0):
+            z = complex(x, y)
+            if abs(z) >= 6:
+                continue
+            w = orc.fast_nuclear_W(z)
+            assert abs(w - wofz(z)) <= 2e-3 * abs(wofz(z)), z
+
+
+def test_faddeeva_asymptotic_region_vs_scipy(orc):
+    for r in (6.0, 7.5, 10.0, 30.0, 100.0):
+        for th in np.linspace(0.02, np.pi - 0.02, 17):
+            z = r * np.exp(1j * th)
+            w = orc.fast_nuclear_W(z)
+            # 2-pole asymptotic expansion: O(1e-5) absolute at |z| = 6
+            assert abs(w - wofz(z)) <= 2e-5, z
+
+
+# ---------------------------------------------------------------- PIN-10
+def test_fast_exp_error_bound(orc):
+    for x in np.linspace(-8, 8, 161):
+        want = np.exp(x)
+        got = orc.fast_exp(x)
+        # (1 + x/n)^n = e^x (1 - x^2/(2n) + O(x^3/n^2)), n = 4096
+        assert abs(got - want) <= (x * x / 8192 * 1.02 + 1e-14) * want, x
+
+
+# ---------------------------------------------------------------- lookups
+@pytest.fixture(scope="module")
+def rs_small():
+    return RS.make_tables(n_nuc=20, avg_poles=60, avg_windows=6)
+
+
+def _macro_bg_only(t, E, mat):
+    want = np.zeros(4)
+    for j in range(int(t["num_nucs"][mat])):
+        n = int(t["mats"][mat, j])
+        nw = int(t["n_windows"][n])
+        w = min(int(E * nw), nw - 1)
+        T, A_, F = (t["windows"][f][n, w] for f in ("T", "A", "F"))
+        want += t["concs"][mat, j] * np.array([E * T, E * A_, E * F, E * T - E * A_])
+    return want
+
+
+def test_background_only_closed_form(orc, rs_small):
+    t = {k: (v.copy() if isinstance(v, np.ndarray) else v) for k, v in rs_small.items()}
+    t["windows"]["end"] = t["windows"]["start"]           # no poles in any window
+    P = orc.RsProblem(t)
+    n = 400
+    out, v, _ = P.run(0, n, X.SEED_L, 1, verify=True)
+    for i, E in enumerate(energies(X.SEED_L, n)):
+        want = _macro_bg_only(t, E, int(v["mat"][i]))
+        np.testing.assert_allclose(v["macro"][i], want, rtol=1e-13, atol=1e-15)
+
+
+def test_single_pole_against_scipy_faddeeva(orc, rs_small):
+    # One pole per window, K0RS = 0 (sigT factor 1), poles mirrored so that
+    # Z = (E - EA)/2 lies in the upper half plane where the approximation is
+    # within ~1e-3 of wofz: the assembled micro XS must match the pole
+    # formula evaluated with scipy's W to that accuracy.
+    t = {k: (v.copy() if isinstance(v, np.ndarray) else v) for k, v in rs_small.items()}
+    t["windows"]["end"] = t["windows"]["start"] + 1
+    t["k0rs"][:] = 0.0
+    t["poles"]["EA"][..., 1] *= -1.0
+    P = orc.RsProblem(t)
+    n = 200
+    out, v, _ = P.run(0, n, X.SEED_L, 1, verify=True)
+    for i, E in enumerate(energies(X.SEED_L, n)):
+        mat = int(v["mat"][i])
+        want = _macro_bg_only(t, E, mat)
+        for j in range(int(t["num_nucs"][mat])):
+            nuc = int(t["mats"][mat, j])
+            nw = int(t["n_windows"][nuc])
+            w = min(int(E * nw), nw - 1)
+            p = t["poles"][nuc, int(t["windows"]["start"][nuc, w])]
+            EA = complex(*p["EA"])
+            W = wofz((E - EA) * 0.5)
+            sT = (complex(*p["RT"]) * W).real
+            sA = (complex(*p["RA"]) * W).real
+            sF = (complex(*p["RF"]) * W).real
+            want += t["concs"][mat, j] * np.array([sT, sA, sF, sT - sA])
+        np.testing.assert_allclose(v["macro"][i], want, rtol=5e-3, atol=1e-3)
+
+
+def test_rs_threads_and_invariants(orc, rs_small):
+    P = orc.RsProblem(rs_small)
+    a, va, ma = P.run(0, 3000, X.SEED_L, 1, verify=True)
+    b, vb, mb = P.run(0, 3000, X.SEED_L, 4, verify=True)
+    assert np.array_equal(a, b) and ma == mb
+    assert np.array_equal(va["macro"], vb["macro"])
+    assert a[0] == sum((k + 1) * int(a[13 + k]) for k in range(4))
+    assert a[1:13].sum() == 3000 and a[13:17].sum() == 3000
+    for i in range(3000):
+        assert int(va["am"][i]) == int(np.argmax(va["macro"][i]))
+    assert ma > 0
+
+
+def test_rs_generator_structure():
+    t = RS.make_tables()
+    assert t["n_poles"].sum() == 355 * 1000 and t["n_windows"].sum() == 355 * 100
+    assert t["poles"].dtype.itemsize == 72 and t["windows"].dtype.itemsize == 32
+    w = t["windows"]
+    for n in (0, 17, 354):
+        nw = int(t["n_windows"][n])
+        assert w["start"][n, 0] == 0
+        assert w["end"][n, nw - 1] == t["n_poles"][n] - 1
