@@ -1,0 +1,366 @@
+"""bench.py -- XSBench lookups/s per mode + fork/join ns, % of HBM roofline.
+
+Metric (BASELINE.json): "XSBench lookups/s per mode + fork/join ns; % HBM
+roofline at 1/2/4/8 B200".  Workload = config 5, XSBench large: 355 nuclides
+x 11,303 gridpoints, 17M lookups per GPU (weak scaling), synthetic seeded
+tables (gtr_inputs).  One step = one batch of 17M lookups through libgtr's
+headline variant (SPMD-ized + heap-to-stack + folding, thread_limit 256 --
+the paper's optimized form of XSBench's `target teams distribute parallel
+for`) plus, for N > 1, the NCCL all-reduce of the 18 u64 hash/tallies.
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--impl gtr|reference]
+    torchrun --nproc-per-node N bench.py --gpus N ...
+
+Rank 0 prints one JSON line.  `--impl reference` times the oracle (plain C on
+the host cores) on a bounded sample of the same workload instead.
+"""
+import argparse
+import json
+import os
+import subprocess
+import sys
+import tempfile
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+N_ISO, N_GP, LOOKUPS_PER_GPU = 355, 11303, 17_000_000
+METRIC = "XSBench lookups/s per mode + fork/join ns; % HBM roofline at 1/2/4/8 B200"
+WORKLOAD = "XSBench large: 355 nuclides x 11,303 gridpoints, 17M lookups per GPU"
+BYTES_PER_NUCLIDE = 100     # 4 B index-grid entry + 2 x 48 B gridpoints
+
+
+def parse():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=10)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", default="gtr", choices=["gtr", "reference"])
+    ap.add_argument("--no-sweep", action="store_true", help="skip the per-mode / fork-join sweeps")
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    return ap.parse_args()
+
+
+# ---------------------------------------------------------------- helpers
+def peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        d = json.load(open(p))
+        return float(d["hbm_gbs"]), "measured"
+    return 6650.0, "fallback"
+
+
+class Clocks:
+    """nvidia-smi sampler for the timed region (B200_PROFILING.md clocks line)."""
+    Q = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+         "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+         "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, gpu):
+        self.gpu = gpu
+        self.f = tempfile.NamedTemporaryFile("w+", suffix=".csv", delete=False)
+        self.p = None
+
+    def __enter__(self):
+        try:
+            self.p = subprocess.Popen(["nvidia-smi", "-i", str(self.gpu), f"--query-gpu={self.Q}",
+                                       "--format=csv,noheader,nounits", "-lms", "100"],
+                                      stdout=self.f, stderr=subprocess.DEVNULL)
+        except OSError:
+            self.p = None
+        time.sleep(0.3)
+        return self
+
+    def __exit__(self, *a):
+        if self.p:
+            self.p.terminate()
+            self.p.wait()
+
+    def summary(self):
+        self.f.flush()
+        rows = [l.split(", ") for l in open(self.f.name).read().strip().splitlines() if l.count(",") >= 8]
+        if not rows:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["unavailable"], "samples": 0}
+        sm = np.array([float(r[1]) for r in rows])
+        smax = float(rows[0][2])
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        reasons = sorted({names[k] for r in rows for k in range(4) if r[5 + k].strip() == "Active"})
+        load = sm[sm >= 0.5 * sm.max()] if sm.max() > 0 else sm
+        return {"sm_mhz": float(np.median(load)), "sm_max_mhz": smax, "reasons": reasons,
+                "samples": len(rows)}
+
+
+def dist_init():
+    import torch
+    ws = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    if ws > 1:
+        import torch.distributed as dist
+        os.environ.setdefault("MASTER_ADDR", "127.0.0.1")
+        torch.cuda.set_device(local)
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    else:
+        torch.cuda.set_device(0)
+    return ws, rank, local
+
+
+def cpu_baseline(tables, first, n, seed):
+    """The oracle as it stands, on the host cores, bounded sample."""
+    import oracle
+    P = oracle.XsProblem(tables)
+    cores = os.cpu_count() or 1
+    t0 = time.perf_counter()
+    out, _ = P.run(first, n, seed, cores)
+    dt = time.perf_counter() - t0
+    return {"value": n / dt, "unit": "lookups/s", "cores": cores, "kind": "oracle",
+            "sample": f"lookups [{first}, {first + n}) of rank 0's range (of {LOOKUPS_PER_GPU}), "
+                      f"{cores} pthreads, table build excluded",
+            "seconds": dt}, out
+
+
+# ---------------------------------------------------------------- reference arm
+def run_reference(a):
+    ws = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return
+    import gtr_inputs.xs as X
+    import oracle
+    t = X.make_tables(N_ISO, N_GP)
+    P = oracle.XsProblem(t)
+    cores = os.cpu_count() or 1
+    sample = 400_000
+    for w in range(a.warmup):
+        P.run(w * sample, sample, X.SEED_L, cores)
+    t0 = time.perf_counter()
+    for s in range(a.steps):
+        P.run(s * sample, sample, X.SEED_L, cores)
+    dt = (time.perf_counter() - t0) / a.steps
+    v = sample / dt
+    line = {"impl": "reference", "metric": METRIC, "value": v, "unit": "lookups/s", "n_gpus": a.gpus,
+            "steps": a.steps, "warmup": a.warmup, "ms_per_step": dt * 1e3, "higher_is_better": True,
+            "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+            "config": {"workload": WORKLOAD, "variant": "C oracle (oracle/xs.c), -O2 -ffp-contract=off",
+                       "sample_per_step": sample},
+            "cpu_baseline": {"value": v, "unit": "lookups/s", "cores": cores, "kind": "oracle",
+                             "sample": f"{sample} lookups per step of the 17M-lookup workload, {cores} pthreads"},
+            "e2e": {"value": v, "unit": "lookups/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+
+
+# ---------------------------------------------------------------- gtr arm
+def run_gtr(a):
+    import torch
+    import gtr_inputs.xs as X
+    from paper_conf_cgo_hubercgtddcd22_b200 import gtr as G
+    from paper_conf_cgo_hubercgtddcd22_b200.problems import XsDevice
+
+    ws, rank, local = dist_init()
+    dist = None
+    if ws > 1:
+        import torch.distributed as dist
+    dev = torch.device("cuda", local)
+    stream = torch.cuda.current_stream()
+    pool = torch.zeros(64 << 20, dtype=torch.uint8, device=dev)
+    ctx = G.gtr_ctx_create(local, pool.data_ptr(), pool.numel())
+
+    t_setup = time.perf_counter()
+    tables = X.make_tables(N_ISO, N_GP)
+    xs = XsDevice(ctx, tables, device=dev)
+    torch.cuda.synchronize()
+    t_setup = time.perf_counter() - t_setup
+    first, n, seed = rank * LOOKUPS_PER_GPU, LOOKUPS_PER_GPU, X.SEED_L
+    head = G.cfg(G.SPMD, G.PL_STACK, 1, 256)
+    out = torch.zeros(18, dtype=torch.uint64, device=dev)
+    num_nucs = tables["num_nucs"].astype(np.int64)
+
+    def step():
+        out.zero_()
+        G.gtr_xs_lookup(ctx, head, xs.tables, first, n, seed, out, None, stream)
+        if dist is not None:
+            dist.all_reduce(out.view(torch.int64), op=dist.ReduceOp.SUM)
+
+    for _ in range(a.warmup):
+        step()
+    G.gtr_ctx_check(ctx, stream)
+
+    # timed region: K steps, barrier + sync on both sides, CUDA events on the
+    # launching stream; per-launch kernel events for the roofline
+    kev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(a.steps)]
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    with Clocks(local) as clk:
+        if dist is not None:
+            dist.barrier()
+        torch.cuda.synchronize()
+        e0.record(stream)
+        for s in range(a.steps):
+            out.zero_()
+            kev[s][0].record(stream)
+            G.gtr_xs_lookup(ctx, head, xs.tables, first, n, seed, out, None, stream)
+            kev[s][1].record(stream)
+            if dist is not None:
+                dist.all_reduce(out.view(torch.int64), op=dist.ReduceOp.SUM)
+        e1.record(stream)
+        torch.cuda.synchronize()
+        if dist is not None:
+            dist.barrier()
+    G.gtr_ctx_check(ctx, stream)
+    ms = e0.elapsed_time(e1) / a.steps
+    k_ms = float(np.mean([b.elapsed_time(c) for b, c in kev]))
+    res = out.cpu().numpy().astype(np.uint64)
+    t_ms = torch.tensor([ms, k_ms], dtype=torch.float64, device=dev)
+    if dist is not None:
+        dist.all_reduce(t_ms, op=dist.ReduceOp.MAX)
+    ms, k_ms = float(t_ms[0]), float(t_ms[1])
+    value = ws * n / (ms * 1e-3)
+
+    # algorithmic bytes of one launch (this rank): sum over sampled materials
+    # of num_nucs x 100 B; the material tallies of all ranks are in `res`
+    mat_tally = res[1:13].astype(np.int64)
+    alg_bytes_all = float((mat_tally * num_nucs).sum() * BYTES_PER_NUCLIDE)
+    alg_bytes = alg_bytes_all / ws
+    hbm, peak_kind = peaks()
+    achieved = alg_bytes / (k_ms * 1e-3) / 1e9
+    traffic = None
+    prof = os.path.join(ROOT, "profiles", "xs_headline_ncu.json")
+    if os.path.exists(prof):
+        traffic = json.load(open(prof)).get("dram_bytes_per_launch")
+
+    extra = {}
+    if rank == 0 and not a.no_sweep:
+        extra = sweeps(G, torch, ctx, xs, first, seed, stream)
+
+    # e2e through the public host-buffer entry point (H2D request, D2H results)
+    h_out = torch.zeros(18, dtype=torch.uint64).pin_memory()
+    req = G.gtr_xs_request(first, n, seed)
+    G.gtr_xs_lookup_host(ctx, head, xs.tables, req, h_out, stream)
+    if dist is not None:
+        dist.barrier()
+    t0 = time.perf_counter()
+    for _ in range(a.steps):
+        G.gtr_xs_lookup_host(ctx, head, xs.tables, req, h_out, stream)
+    e2e_s = (time.perf_counter() - t0) / a.steps
+    t_e = torch.tensor([e2e_s], dtype=torch.float64, device=dev)
+    if dist is not None:
+        dist.all_reduce(t_e, op=dist.ReduceOp.MAX)
+    e2e_s = float(t_e[0])
+
+    cpu = None
+    parity = None
+    if rank == 0 and ws == 1 and not a.no_cpu_baseline:
+        m = 2_000_000
+        cpu, o_out = cpu_baseline(tables, first, m, seed)
+        chk = torch.zeros(18, dtype=torch.uint64, device=dev)
+        G.gtr_xs_lookup(ctx, head, xs.tables, first, m, seed, chk, None, stream)
+        parity = bool(np.array_equal(chk.cpu().numpy(), o_out))
+        cpu.pop("seconds")
+
+    if rank == 0:
+        line = {
+            "metric": METRIC, "value": value, "unit": "lookups/s", "n_gpus": ws, "steps": a.steps,
+            "warmup": a.warmup, "ms_per_step": ms, "higher_is_better": True, "scaling": "weak",
+            "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+            "config": {"workload": WORKLOAD, "variant": "SPMD + heap-to-stack + folding, thread_limit 256",
+                       "lookups_per_gpu": n, "parallelism": f"lookups sharded over {ws} GPU(s), NCCL all-reduce "
+                                                             "of hash+tallies" if ws > 1 else "1 GPU",
+                       "l2": "no flush: inputs 5.9 GB per GPU >> 126 MB L2 (index grid 5.7 GB)",
+                       "table_setup_s": round(t_setup, 2)},
+            "hash": int(res[0]), "hash_mod_999983": int(res[0] % 999983),
+            "roofline": {"bound": "hbm", "achieved": achieved, "peak": hbm, "unit": "GB/s",
+                         "frac": achieved / hbm, "traffic": traffic,
+                         "kernel_ms": k_ms, "alg_bytes_per_launch": alg_bytes,
+                         "peak_source": f"{peak_kind} MEASURED_PEAKS.json hbm_gbs" if peak_kind == "measured"
+                         else "fallback B200_PROFILING.md 6.65 TB/s"},
+            "cpu_baseline": cpu, "parity_vs_oracle_2M_sample": parity,
+            "e2e": {"value": ws * n / e2e_s, "unit": "lookups/s",
+                    "h2d_bytes_per_step": 24, "d2h_bytes_per_step": 144,
+                    "note": "gtr_xs_lookup_host: pinned host request -> device, lookups, 18 u64 -> pinned host, "
+                            "stream sync; tables resident (uploaded once, table_setup_s)"},
+            "gpu_launches": a.steps,
+            "clocks": clk.summary(),
+        }
+        line.update(extra)
+        print(json.dumps(line), flush=True)
+    G.gtr_ctx_destroy(ctx)
+    if dist is not None:
+        dist.destroy_process_group()
+
+
+def _time(torch, stream, fn, reps):
+    fn()
+    torch.cuda.synchronize()
+    a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    a.record(stream)
+    for _ in range(reps):
+        fn()
+    b.record(stream)
+    torch.cuda.synchronize()
+    return a.elapsed_time(b) / reps
+
+
+def sweeps(G, torch, ctx, xs, first, seed, stream):
+    """Per-mode lookups/s (same 17M lookups), the paper's variant ladder, and
+    fork/join ns per mode -- each checked for identical results."""
+    n = LOOKUPS_PER_GPU
+    out = torch.zeros(18, dtype=torch.uint64, device="cuda")
+    modes = {}
+    ref = None
+    for name, c in [("native", G.cfg(G.NATIVE, G.PL_STACK, 1, 256)),
+                    ("spmd", G.cfg(G.SPMD, G.PL_STACK, 1, 256)),
+                    ("csm", G.cfg(G.CSM, G.PL_STACK, 1, 256)),
+                    ("cascade", G.cfg(G.GENERIC_CASCADE, G.PL_STACK, 1, 256)),
+                    ("generic", G.cfg(G.GENERIC, G.PL_STACK, 1, 256))]:
+        def f():
+            out.zero_()
+            G.gtr_xs_lookup(ctx, c, xs.tables, first, n, seed, out, None, stream)
+        ms = _time(torch, stream, f, 3)
+        r = out.cpu().numpy()
+        ref = r if ref is None else ref
+        info = G.gtr_query_variant(G.K_XS, c)
+        modes[name] = {"lookups_per_s": n / (ms * 1e-3), "ms": ms, "regs": info["regs"],
+                       "static_smem": info["static_smem"], "dyn_smem": info["dyn_smem"],
+                       "teams_per_sm": info["teams_per_sm"], "same_result": bool(np.array_equal(r, ref))}
+    # the paper's ladder (Fig. 11a) on SPMD: globalized at runtime -> h2s2 -> +fold
+    ladder = {}
+    for name, c in [("runtime_globalized", G.cfg(G.SPMD, G.PL_RUNTIME, 0, 256)),
+                    ("global_heap", G.cfg(G.SPMD, G.PL_GLOBAL, 0, 256)),
+                    ("heap_to_shared", G.cfg(G.SPMD, G.PL_SHARED_STATIC, 0, 256)),
+                    ("heap_to_stack", G.cfg(G.SPMD, G.PL_STACK, 0, 256)),
+                    ("heap_to_stack_fold", G.cfg(G.SPMD, G.PL_STACK, 1, 256))]:
+        def f():
+            out.zero_()
+            G.gtr_xs_lookup(ctx, c, xs.tables, first, n, seed, out, None, stream)
+        ms = _time(torch, stream, f, 2)
+        ladder[name] = {"lookups_per_s": n / (ms * 1e-3), "ms": ms,
+                        "same_result": bool(np.array_equal(out.cpu().numpy(), ref))}
+    G.gtr_ctx_check(ctx, stream)
+    # fork/join ns: 148 teams (one per SM), 20,000 trivial regions, K = 4
+    fj = {}
+    R, teams = 20000, 148
+    fo = torch.zeros(teams, dtype=torch.uint64, device="cuda")
+    for nt in (128, 256):
+        row = {}
+        fl = G.cfg(thread_limit=nt, num_teams=teams)
+        row["barrier_floor_ns"] = _time(torch, stream, lambda: G.gtr_barrier_floor(ctx, fl, R, fo, stream), 2) \
+            * 1e6 / R
+        for name, m, flags in [("generic", G.GENERIC, 0), ("cascade", G.GENERIC_CASCADE, 0),
+                               ("csm", G.CSM, 0), ("spmd", G.SPMD, 0)]:
+            c = G.cfg(m, G.PL_SHARED_STATIC, 1, nt, num_teams=teams, flags=flags)
+            ms = _time(torch, stream, lambda: G.gtr_forkjoin(ctx, c, R, 1, 4, fo, stream), 2)
+            row[name + "_ns"] = ms * 1e6 / R
+            row[name + "_regs"] = G.gtr_query_variant(G.K_FORKJOIN, c)["regs"]
+        fj[f"thread_limit_{nt}"] = row
+    G.gtr_ctx_check(ctx, stream)
+    return {"modes": modes, "ladder_spmd": ladder, "forkjoin": fj}
+
+
+if __name__ == "__main__":
+    a = parse()
+    if a.impl == "reference":
+        run_reference(a)
+    else:
+        run_gtr(a)

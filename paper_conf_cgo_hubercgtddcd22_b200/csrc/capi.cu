@@ -1,0 +1,93 @@
+// capi.cu -- context management, status strings and variant queries of the
+// C ABI declared in include/gtr.h.
+#include <cstdlib>
+
+#include "gtr_internal.h"
+
+using namespace gtr;
+
+extern "C" int gtr_version(void) { return GTR_VERSION; }
+
+extern "C" const char *gtr_strerror(int status) {
+    switch (status) {
+    case GTR_OK: return "ok";
+    case GTR_EINVAL: return "invalid argument or configuration";
+    case GTR_ECUDA: return "CUDA runtime error";
+    case GTR_ENOMEM: return "workspace or pool too small";
+    case GTR_EHEAP: return "device fallback heap exhausted (globalized variables did not fit)";
+    case GTR_EDEVICE: return "device-side error flag set";
+    case GTR_EUNSUPPORTED: return "configuration not instantiated";
+    default: return "unknown status";
+    }
+}
+
+extern "C" int gtr_ctx_create(int device, void *fallback_pool, uint64_t fallback_pool_bytes, gtr_ctx **out) {
+    if (!out) return GTR_EINVAL;
+    *out = nullptr;
+    int n = 0;
+    GTR_CUDA_TRY(cudaGetDeviceCount(&n));
+    if (device < 0 || device >= n) return GTR_EINVAL;
+    GTR_CUDA_TRY(cudaSetDevice(device));
+    gtr_ctx *c = static_cast<gtr_ctx *>(calloc(1, sizeof(gtr_ctx)));
+    if (!c) return GTR_ENOMEM;
+    c->device = device;
+    if (cudaDeviceGetAttribute(&c->num_sms, cudaDevAttrMultiProcessorCount, device) != cudaSuccess ||
+        cudaMalloc(&c->d_err, 256) != cudaSuccess || cudaMalloc(&c->d_stage, 256) != cudaSuccess ||
+        cudaMemset(c->d_err, 0, 256) != cudaSuccess) {
+        if (c->d_err) cudaFree(c->d_err);
+        if (c->d_stage) cudaFree(c->d_stage);
+        free(c);
+        return GTR_ECUDA;
+    }
+    c->pool = static_cast<uint64_t *>(fallback_pool);
+    c->pool_bytes = fallback_pool ? fallback_pool_bytes : 0;
+    *out = c;
+    return GTR_OK;
+}
+
+extern "C" int gtr_ctx_destroy(gtr_ctx *c) {
+    if (!c) return GTR_EINVAL;
+    cudaFree(c->d_err);
+    cudaFree(c->d_stage);
+    free(c);
+    return GTR_OK;
+}
+
+extern "C" int gtr_ctx_check(gtr_ctx *c, void *stream) {
+    if (!c) return GTR_EINVAL;
+    cudaStream_t s = static_cast<cudaStream_t>(stream);
+    uint32_t err = 0;
+    GTR_CUDA_TRY(cudaMemcpyAsync(&err, c->d_err, sizeof(err), cudaMemcpyDeviceToHost, s));
+    GTR_CUDA_TRY(cudaStreamSynchronize(s));
+    GTR_CUDA_TRY(cudaGetLastError());
+    if (err == 0) return GTR_OK;
+    GTR_CUDA_TRY(cudaMemsetAsync(c->d_err, 0, sizeof(err), s));
+    GTR_CUDA_TRY(cudaStreamSynchronize(s));
+    if (err & ERR_HEAP) return GTR_EHEAP;
+    return GTR_EDEVICE;
+}
+
+// family query hooks (each family's TU)
+int gtr_internal_query_xs(gtr_ctx *, const gtr_launch_cfg *, gtr_variant_info *);
+int gtr_internal_query_su3(gtr_ctx *, const gtr_launch_cfg *, gtr_variant_info *);
+int gtr_internal_query_rs(gtr_ctx *, const gtr_launch_cfg *, gtr_variant_info *);
+int gtr_internal_query_fj(gtr_ctx *, const gtr_launch_cfg *, gtr_variant_info *, int floor);
+int gtr_internal_query_sem(gtr_ctx *, const gtr_launch_cfg *, gtr_variant_info *);
+
+extern "C" int gtr_query_variant(int kernel, const gtr_launch_cfg *cfg, gtr_variant_info *out) {
+    if (!cfg || !out) return GTR_EINVAL;
+    gtr_ctx tmp = {};
+    int dev = 0;
+    GTR_CUDA_TRY(cudaGetDevice(&dev));
+    tmp.device = dev;
+    GTR_CUDA_TRY(cudaDeviceGetAttribute(&tmp.num_sms, cudaDevAttrMultiProcessorCount, dev));
+    switch (kernel) {
+    case GTR_K_XS: return gtr_internal_query_xs(&tmp, cfg, out);
+    case GTR_K_SU3: return gtr_internal_query_su3(&tmp, cfg, out);
+    case GTR_K_RS: return gtr_internal_query_rs(&tmp, cfg, out);
+    case GTR_K_FORKJOIN: return gtr_internal_query_fj(&tmp, cfg, out, 0);
+    case GTR_K_BARRIER_FLOOR: return gtr_internal_query_fj(&tmp, cfg, out, 1);
+    case GTR_K_SEMANTICS: return gtr_internal_query_sem(&tmp, cfg, out);
+    default: return GTR_EINVAL;
+    }
+}

@@ -1,0 +1,131 @@
+// gtr_internal.h -- host-side helpers shared by the kernel translation units
+// (context, launch-configuration resolution, variant dispatch).
+#pragma once
+#include <cstdint>
+#include <cstdio>
+#include <cuda_runtime.h>
+
+#include "../../include/gtr.h"
+#include "gtr_rt.cuh"
+
+struct gtr_ctx {
+    int device;
+    int num_sms;
+    uint64_t *pool;
+    uint64_t pool_bytes;
+    uint32_t *d_err;       // device error word
+    void *d_stage;         // 256 B staging buffer (e2e request / results)
+};
+
+namespace gtr {
+
+#define GTR_CUDA_TRY(x)                                                                    \
+    do {                                                                                   \
+        cudaError_t e_ = (x);                                                              \
+        if (e_ != cudaSuccess) {                                                           \
+            if (getenv("GTR_DEBUG")) fprintf(stderr, "gtr: %s:%d %s\n", __FILE__, __LINE__, \
+                                             cudaGetErrorString(e_));                      \
+            return GTR_ECUDA;                                                              \
+        }                                                                                  \
+    } while (0)
+
+// Resolved launch geometry for one variant.
+struct Launch {
+    int block;          // hardware threads per CTA
+    int teams;          // grid size
+    uint32_t dyn_smem;  // dynamic shared memory bytes
+    RtParams rp;
+};
+
+inline uint32_t odd_words(uint32_t bytes) {
+    uint32_t w = (bytes + 7u) / 8u;
+    return (w % 2u == 1u) ? w : w + 1u;
+}
+
+// Compute geometry + runtime params for variant K of kernel `fn`.
+template <class K>
+int resolve(gtr_ctx *ctx, const gtr_launch_cfg *cfg, const void *fn, uint32_t default_stack_bytes,
+            Launch *L, bool stack_always = false) {
+    L->block = K::BLOCK;
+    uint32_t stack_words = 0, stride = 0;
+    if (K::PL == PL_RUNTIME || (stack_always && K::PL != PL_GLOBAL)) {
+        uint32_t bytes = cfg->smem_stack_bytes ? cfg->smem_stack_bytes : default_stack_bytes;
+        stack_words = (bytes + 7u) / 8u;
+        if (stack_words > 4095u) return GTR_EINVAL;
+        stride = odd_words(bytes);
+    }
+    L->dyn_smem = tstate_bytes<K>() + (uint32_t)K::BLOCK * stride * 8u;
+    if (L->dyn_smem > 48u * 1024u) {
+        if (cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)L->dyn_smem) !=
+            cudaSuccess)
+            return GTR_EINVAL;
+    }
+    int per_sm = 0;
+    GTR_CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, fn, K::BLOCK, L->dyn_smem));
+    if (per_sm < 1) return GTR_EINVAL;
+    L->teams = cfg->num_teams > 0 ? cfg->num_teams : per_sm * ctx->num_sms;
+    L->rp.err = ctx->d_err;
+    L->rp.pool = ctx->pool;
+    uint64_t hw = (uint64_t)L->teams * (uint64_t)K::BLOCK;
+    L->rp.pool_wpt = ctx->pool ? (ctx->pool_bytes / 8u) / hw : 0;
+    L->rp.sm_stack_words = stack_words;
+    L->rp.sm_stride_words = stride;
+    return GTR_OK;
+}
+
+template <class K> int fill_info(const void *fn, const Launch &L, int per_sm, gtr_variant_info *out) {
+    cudaFuncAttributes a;
+    GTR_CUDA_TRY(cudaFuncGetAttributes(&a, fn));
+    out->regs = a.numRegs;
+    out->static_smem = (int32_t)a.sharedSizeBytes;
+    out->dyn_smem = (int32_t)L.dyn_smem;
+    out->local_bytes = (int32_t)a.localSizeBytes;
+    out->block_threads = L.block;
+    out->teams_per_sm = per_sm;
+    out->num_teams = L.teams;
+    return GTR_OK;
+}
+
+// Variant dispatch: Op<K>::run(args...) for the runtime (mode, placement,
+// fold, thread_limit) triple; NATIVE handled by the caller.
+template <int NT, int FLAGS, template <class> class Op, class... A>
+int dispatch_mpf(int mode, int pl, int fold, A &&...a) {
+#define GTR_CASE(M, P)                                                                     \
+    if (mode == M && pl == P) {                                                            \
+        if (fold) return Op<Cfg<M, P, true, NT, FLAGS>>::run(a...);                        \
+        return Op<Cfg<M, P, false, NT, FLAGS>>::run(a...);                                 \
+    }
+#define GTR_CASES(M)                                                                       \
+    GTR_CASE(M, PL_RUNTIME) GTR_CASE(M, PL_GLOBAL) GTR_CASE(M, PL_SHARED_STATIC) GTR_CASE(M, PL_STACK)
+    GTR_CASES(GENERIC)
+    GTR_CASES(GENERIC_CASCADE)
+    GTR_CASES(CSM)
+    GTR_CASES(SPMD)
+#undef GTR_CASES
+#undef GTR_CASE
+    return GTR_EUNSUPPORTED;
+}
+
+// SPMD-only dispatch (flags that only change SPMD-ized code).
+template <int NT, int FLAGS, template <class> class Op, class... A>
+int dispatch_spmd(int pl, int fold, A &&...a) {
+#define GTR_CASE(P)                                                                        \
+    if (pl == P) {                                                                         \
+        if (fold) return Op<Cfg<SPMD, P, true, NT, FLAGS>>::run(a...);                     \
+        return Op<Cfg<SPMD, P, false, NT, FLAGS>>::run(a...);                              \
+    }
+    GTR_CASE(PL_RUNTIME) GTR_CASE(PL_GLOBAL) GTR_CASE(PL_SHARED_STATIC) GTR_CASE(PL_STACK)
+#undef GTR_CASE
+    return GTR_EUNSUPPORTED;
+}
+
+inline bool valid_cfg(const gtr_launch_cfg *c) {
+    if (!c) return false;
+    if (c->mode < 0 || c->mode > 4) return false;
+    if (c->placement < 0 || c->placement > 3) return false;
+    if (c->thread_limit <= 0 || c->thread_limit % 32 != 0) return false;
+    if (c->num_teams < 0) return false;
+    return true;
+}
+
+}  // namespace gtr

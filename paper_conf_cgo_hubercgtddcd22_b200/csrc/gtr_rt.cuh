@@ -1,0 +1,444 @@
+// gtr_rt.cuh -- the GPU team runtime: CPU-style OpenMP execution on a CTA.
+//
+// Device-side counterpart of the paper's "device runtime, roughly the GPU
+// equivalent of the host OpenMP runtime" and of the kernel
+// shapes its LLVM optimizations produce (Section IV).  Written for
+// sm_100a; header-only, included by every kernel translation unit.
+//
+//   team = CTA, OpenMP thread = hardware thread        (Fig. 2)
+//   GENERIC          main thread + worker state machine, regions passed as
+//                    function pointers, workers call indirectly
+//   GENERIC_CASCADE  workers compare the pointer against the known regions
+//                    and call them directly, indirect fallback
+//   CSM              custom state machine: region IDs, direct calls only, no
+//                    address-taken region functions (fn. 4)
+//   SPMD             SPMD-ized: all threads run the team code; side effects
+//                    guarded by thread 0 + barrier, values broadcast through
+//                    shared memory (Fig. 7)
+//   NATIVE           plain CUDA (the paper's CUDA watermark);
+//                    kernels written without this runtime.
+//
+// Globalization: Local<> / TeamLocal<> realise each globalized
+// variable in one of four placements --
+//   PL_RUNTIME        __runtime_alloc: per-thread LIFO stack in dynamic shared
+//                     memory, global-memory fallback pool
+//   PL_GLOBAL         the fallback only (shared stack of size 0; the paper's
+//                     "LIBOMPTARGET_HEAP_SIZE" configuration)
+//   PL_SHARED_STATIC  heap-to-shared: static __shared__ storage;
+//                     per-thread variables scaled by the thread count (Fig. 6b)
+//   PL_STACK          heap-to-stack: registers / local memory
+//
+// Runtime-call folding: with FOLD the execution-mode, parallel-
+// level, thread-count and launch-parameter queries are compile-time constants;
+// without it they read the team/thread state in shared memory.
+#pragma once
+#include <cstdint>
+#include <cuda_runtime.h>
+
+namespace gtr {
+
+enum : int { GENERIC = 0, GENERIC_CASCADE = 1, CSM = 2, SPMD = 3, NATIVE = 4 };
+enum : int { PL_RUNTIME = 0, PL_GLOBAL = 1, PL_SHARED_STATIC = 2, PL_STACK = 3 };
+enum : uint32_t { ERR_HEAP = 1u, ERR_LIFO = 2u, ERR_DUP_ENERGY = 4u, ERR_BUILD = 8u };
+enum : int { F_BCAST_1BAR = 1, F_SEPARATE_GUARDS = 2 };
+
+// Compile-time kernel configuration.
+template <int MODE_, int PL_, bool FOLD_, int NT_, int FLAGS_ = 0>
+struct Cfg {
+    static constexpr int MODE = MODE_, PL = PL_, NT = NT_, FLAGS = FLAGS_;
+    static constexpr bool FOLD = FOLD_;
+    static constexpr bool GENERIC_LIKE = (MODE_ <= CSM);
+    // generic mode: NT workers + one extra warp whose lane 0 is the main thread
+    static constexpr int BLOCK = GENERIC_LIKE ? NT_ + 32 : NT_;
+    static constexpr int MAIN_HW = GENERIC_LIKE ? NT_ : 0;
+    // per-thread runtime state (stack tops, nesting) lives in dynamic shared
+    // memory for every variant: a STACK/SHARED_STATIC kernel may still make
+    // runtime allocations for variables heap-to-stack could not move (Fig. 6b)
+    static constexpr bool TSTATE = true;
+    static_assert(NT_ % 32 == 0 && NT_ >= 32 && NT_ <= 1024 - (GENERIC_LIKE ? 32 : 0), "bad NT");
+};
+
+// Launch-time runtime parameters (host-filled, by value).
+struct RtParams {
+    uint32_t *err;              // device error word (ctx-owned)
+    uint64_t *pool;             // global fallback pool (caller-owned), may be null
+    uint64_t pool_wpt;          // fallback capacity per hardware thread, 8-byte words
+    uint32_t sm_stack_words;    // shared-memory stack capacity per thread (words)
+    uint32_t sm_stride_words;   // per-thread stride of the stack (odd => no bank conflicts)
+};
+
+typedef void (*RegionFn)(void *);
+
+// Team state, one per CTA (static shared memory).
+struct TeamState {
+    RegionFn volatile fn;       // work descriptor (GENERIC / CASCADE)
+    void *volatile args;
+    volatile int32_t region_id; // work descriptor (CSM); 0 = terminate
+    volatile int32_t level;     // team parallel level seen by workers (generic)
+    volatile int32_t nthreads;  // threads of the active parallel region
+    int32_t exec_mode;          // ICV read by non-folded is_spmd()
+    RtParams rp;
+    uint64_t bcast[2];          // guarded-value broadcast slots
+};
+static __shared__ TeamState g_ts;
+
+// Per-thread state (dynamic shared memory, offset 0) -- only when TSTATE.
+struct ThreadState {
+    uint16_t sp;      // shared stack top (words)
+    uint8_t nested;   // serialized nested parallel depth
+    uint8_t level;    // SPMD: this thread's parallel level
+    uint32_t gsp;     // global fallback stack top (words)
+};
+extern __shared__ __align__(16) uint8_t g_dyn[];
+
+template <class K> __host__ __device__ constexpr uint32_t tstate_bytes() {
+    return K::TSTATE ? (uint32_t)((K::BLOCK * sizeof(ThreadState) + 15) / 16 * 16) : 0u;
+}
+template <class K> __device__ __forceinline__ ThreadState &tstate() {
+    return reinterpret_cast<ThreadState *>(g_dyn)[threadIdx.x];
+}
+template <class K> __device__ __forceinline__ uint64_t *sm_stack_base() {
+    return reinterpret_cast<uint64_t *>(g_dyn + tstate_bytes<K>());
+}
+
+// ---------------------------------------------------------------- barriers
+// Generic mode: the main thread arrives from divergent code while lanes
+// 1..31 of its warp have exited; the non-aligned barrier.sync counts the
+// team (NT workers + 1 warp).  SPMD: plain CTA barrier.
+template <class K> __device__ __forceinline__ void team_barrier() {
+    if constexpr (K::GENERIC_LIKE)
+        asm volatile("barrier.sync 1, %0;" ::"n"(K::BLOCK) : "memory");
+    else
+        __syncthreads();
+}
+
+// `#pragma omp barrier` inside a parallel region: the region's threads only
+// (generic: the NT workers on named barrier 2; the main thread waits at the
+// join).  SPMD: the whole CTA.
+template <class K> __device__ __forceinline__ void omp_barrier() {
+    if constexpr (K::GENERIC_LIKE)
+        asm volatile("barrier.sync 2, %0;" ::"n"(K::NT) : "memory");
+    else
+        __syncthreads();
+}
+
+// Team-wide sync of SPMD-ized sequential code (e.g. before a shared team
+// variable read by all threads is overwritten); generic: no-op (only the main
+// thread runs sequential code).
+template <class K> __device__ __forceinline__ void spmd_sync() {
+    if constexpr (K::MODE == SPMD) __syncthreads();
+}
+
+// ---------------------------------------------------------------- queries
+template <class K> __device__ __forceinline__ int team_num() { return blockIdx.x; }
+template <class K> __device__ __forceinline__ int num_teams() { return gridDim.x; }
+template <class K> __device__ __forceinline__ int warp_size() { return 32; }
+template <class K> __device__ __forceinline__ int warp_id() { return threadIdx.x >> 5; }
+
+template <class K> __device__ __forceinline__ bool is_spmd() {
+    if constexpr (K::FOLD) return K::MODE == SPMD;
+    else return g_ts.exec_mode == SPMD;
+}
+// Folded queries assume the region context the analysis proved:
+// thread/team-count queries are only folded inside parallel regions.
+template <class K> __device__ __forceinline__ int parallel_level() {
+    if constexpr (K::FOLD) return 1;
+    else if constexpr (K::MODE == SPMD) return tstate<K>().level + tstate<K>().nested;
+    else return (threadIdx.x == K::MAIN_HW ? 0 : g_ts.level) + tstate<K>().nested;
+}
+template <class K> __device__ __forceinline__ bool in_active_parallel() {
+    return parallel_level<K>() == 1 && (K::FOLD || tstate<K>().nested == 0);
+}
+template <class K> __device__ __forceinline__ int thread_num() {
+    if constexpr (K::FOLD) return threadIdx.x;
+    else return (parallel_level<K>() == 0 || tstate<K>().nested) ? 0 : (int)threadIdx.x;
+}
+template <class K> __device__ __forceinline__ int num_threads() {
+    if constexpr (K::FOLD) return K::NT;
+    else return (parallel_level<K>() == 0 || tstate<K>().nested) ? 1 : g_ts.nthreads;
+}
+
+// ---------------------------------------------------------------- roles
+enum class Role { Main, Worker, Exit };
+
+// team_init: every hardware thread calls it first.  Generic: lanes 1..31 of
+// the main warp exit, workers must then call worker_loop, the main thread
+// runs the team's sequential code.  SPMD: everybody is Main (runs the team
+// code, guarded).
+template <class K> __device__ __forceinline__ Role team_init(const RtParams &rp) {
+    if constexpr (K::TSTATE) {
+        ThreadState z = {0, 0, 0, 0};
+        tstate<K>() = z;
+    }
+    if constexpr (K::GENERIC_LIKE) {
+        if ((int)threadIdx.x >= K::NT) {
+            if ((int)threadIdx.x != K::MAIN_HW) return Role::Exit;
+            g_ts.fn = nullptr;
+            g_ts.args = nullptr;
+            g_ts.region_id = 0;
+            g_ts.level = 0;
+            g_ts.nthreads = K::NT;
+            g_ts.exec_mode = K::MODE;
+            g_ts.rp = rp;
+            return Role::Main;
+        }
+        return Role::Worker;
+    } else {
+        if (threadIdx.x == 0) {
+            g_ts.level = 0;
+            g_ts.nthreads = K::NT;
+            g_ts.exec_mode = K::MODE;
+            g_ts.rp = rp;
+        }
+        __syncthreads();
+        return Role::Main;
+    }
+}
+
+// ---------------------------------------------------------------- fork/join
+// Region types: struct R { static constexpr int ID = ...; static __device__ void run(void*); }
+template <class K, class R> __device__ __forceinline__ void parallel(void *args) {
+    if constexpr (!K::FOLD) {
+        if (parallel_level<K>() > 0) {          // nested: serialize
+            tstate<K>().nested++;
+            R::run(args);
+            tstate<K>().nested--;
+            return;
+        }
+    }
+    if constexpr (K::MODE == SPMD) {
+        if constexpr (!K::FOLD) tstate<K>().level = 1;
+        R::run(args);                            // in place, all threads
+        if constexpr (!K::FOLD) tstate<K>().level = 0;
+        __syncthreads();                         // join
+    } else {
+        static_assert(K::GENERIC_LIKE, "parallel() needs a runtime mode");
+        if constexpr (K::MODE == CSM)
+            g_ts.region_id = R::ID;
+        else
+            g_ts.fn = &R::run;                   // address taken: GEN / CAS
+        g_ts.args = args;
+        g_ts.level = 1;
+        team_barrier<K>();                       // fork
+        team_barrier<K>();                       // join
+        g_ts.level = 0;
+    }
+}
+
+template <class K, class... Rs> struct Dispatch;
+template <class K> struct Dispatch<K> {
+    static __device__ __forceinline__ bool csm(int, void *) { return false; }
+    static __device__ __forceinline__ bool cascade(RegionFn, void *) { return false; }
+};
+template <class K, class R, class... Rs> struct Dispatch<K, R, Rs...> {
+    static __device__ __forceinline__ bool csm(int id, void *a) {
+        if (id == R::ID) { R::run(a); return true; }
+        return Dispatch<K, Rs...>::csm(id, a);
+    }
+    static __device__ __forceinline__ bool cascade(RegionFn fn, void *a) {
+        if (fn == &R::run) { R::run(a); return true; }
+        return Dispatch<K, Rs...>::cascade(fn, a);
+    }
+};
+
+// The worker state machine.  Regions... are the parallel regions
+// known to reach this kernel (used by CASCADE and CSM; GENERIC ignores them).
+template <class K, class... Rs> __device__ void worker_loop() {
+    for (;;) {
+        team_barrier<K>();                       // wait for work
+        void *a = g_ts.args;
+        if constexpr (K::MODE == CSM) {
+            int id = g_ts.region_id;
+            if (id == 0) return;
+            Dispatch<K, Rs...>::csm(id, a);      // direct calls, no fallback
+        } else {
+            RegionFn fn = g_ts.fn;
+            if (fn == nullptr) return;
+            if constexpr (K::MODE == GENERIC_CASCADE) {
+                if (!Dispatch<K, Rs...>::cascade(fn, a)) fn(a);   // indirect fallback
+            } else {
+                fn(a);                           // indirect call
+            }
+        }
+        team_barrier<K>();                       // join
+    }
+}
+
+template <class K> __device__ __forceinline__ void team_deinit() {
+    if constexpr (K::GENERIC_LIKE) {             // main thread: release workers
+        g_ts.fn = nullptr;
+        g_ts.region_id = 0;
+        team_barrier<K>();
+    }
+}
+
+// ---------------------------------------------------------------- guards
+// SPMD-ized sequential side effects.  Generic modes: only the
+// main thread executes sequential code, so the guard is the identity.
+template <class K, class F> __device__ __forceinline__ void guarded(F &&f) {
+    if constexpr (K::MODE == SPMD) {
+        if (threadIdx.x == 0) f();
+        __syncthreads();
+    } else {
+        f();
+    }
+}
+// A value produced in a guarded region, broadcast to all threads.  Default:
+// slot write -> barrier -> read -> barrier (the paper's 2 barriers,
+// P:687-688).  F_BCAST_1BAR: double-buffered slot, one barrier (`phase`
+// must alternate between consecutive calls).
+template <class K, class T, class F> __device__ __forceinline__ T guarded_bcast(F &&f, int phase = 0) {
+    static_assert(sizeof(T) <= 8, "broadcast slot is 8 bytes");
+    if constexpr (K::MODE == SPMD) {
+        int b = (K::FLAGS & F_BCAST_1BAR) ? (phase & 1) : 0;
+        if (threadIdx.x == 0) *reinterpret_cast<T *>(&g_ts.bcast[b]) = f();
+        __syncthreads();
+        T v = *reinterpret_cast<volatile T *>(&g_ts.bcast[b]);
+        if constexpr (!(K::FLAGS & F_BCAST_1BAR)) __syncthreads();
+        return v;
+    } else {
+        return f();
+    }
+}
+
+// ---------------------------------------------------------------- globalization
+// __runtime_alloc / __runtime_free (Fig. 4c): per-thread LIFO stack in dynamic
+// shared memory; when full, the thread's slab of the global fallback pool; when
+// that is exhausted, ERR_HEAP and a per-CTA sink (results declared invalid).
+__device__ __align__(16) static uint64_t g_sink_dummy;
+template <class K> __device__ __noinline__ void *alloc_shared(uint32_t bytes) {
+    const uint32_t words = (bytes + 7u) >> 3;
+    ThreadState &ts = tstate<K>();
+    const RtParams &rp = g_ts.rp;
+    if constexpr (K::PL == PL_RUNTIME) {
+        if ((uint32_t)ts.sp + words <= rp.sm_stack_words) {
+            uint64_t *p = sm_stack_base<K>() + (size_t)threadIdx.x * rp.sm_stride_words + ts.sp;
+            ts.sp = (uint16_t)(ts.sp + words);
+            return p;
+        }
+    }
+    if (rp.pool != nullptr && (uint64_t)ts.gsp + words <= rp.pool_wpt) {
+        uint64_t *p = rp.pool + ((uint64_t)blockIdx.x * K::BLOCK + threadIdx.x) * rp.pool_wpt + ts.gsp;
+        ts.gsp += words;
+        return p;
+    }
+    atomicOr(rp.err, (uint32_t)ERR_HEAP);
+    return &g_sink_dummy;
+}
+template <class K> __device__ __noinline__ void free_shared(void *p, uint32_t bytes) {
+    const uint32_t words = (bytes + 7u) >> 3;
+    ThreadState &ts = tstate<K>();
+    if (p == &g_sink_dummy) return;
+    if (__isShared(p)) {
+        ts.sp = (uint16_t)(ts.sp - words);
+        if ((uint64_t *)p != sm_stack_base<K>() + (size_t)threadIdx.x * g_ts.rp.sm_stride_words + ts.sp)
+            atomicOr(g_ts.rp.err, (uint32_t)ERR_LIFO);
+    } else {
+        ts.gsp -= words;
+    }
+}
+
+template <int N_WORDS> struct OddStride {
+    static constexpr int value = (N_WORDS % 2 == 1) ? N_WORDS : N_WORDS + 1;
+};
+
+// A per-thread globalized local of N elements of T (8-byte T for the
+// interleaving arithmetic; other sizes round up to whole words).
+template <class K, class T, int N, class Tag, int PL = K::PL> struct Local;
+
+template <class K, class T, int N, class Tag> struct Local<K, T, N, Tag, PL_STACK> {
+    T v[N];
+    __device__ __forceinline__ T &operator[](int i) { return v[i]; }
+    __device__ __forceinline__ T *ptr() { return v; }
+};
+template <class K, class T, int N, class Tag> struct Local<K, T, N, Tag, PL_RUNTIME> {
+    T *p;
+    __device__ __forceinline__ Local() { p = static_cast<T *>(alloc_shared<K>(N * sizeof(T))); }
+    __device__ __forceinline__ ~Local() { free_shared<K>(p, N * sizeof(T)); }
+    __device__ __forceinline__ T &operator[](int i) { return p[i]; }
+    __device__ __forceinline__ T *ptr() { return p; }
+};
+template <class K, class T, int N, class Tag> struct Local<K, T, N, Tag, PL_GLOBAL>
+    : Local<K, T, N, Tag, PL_RUNTIME> {};
+template <class K, class T, int N, class Tag> struct Local<K, T, N, Tag, PL_SHARED_STATIC> {
+    static constexpr int WORDS = (int)((N * sizeof(T) + 7) / 8);
+    static constexpr int STRIDE = OddStride<WORDS>::value;
+    T *p;
+    __device__ __forceinline__ Local() {
+        __shared__ uint64_t slots[K::BLOCK * STRIDE];     // one instance per Tag
+        p = reinterpret_cast<T *>(&slots[threadIdx.x * STRIDE]);
+    }
+    __device__ __forceinline__ T &operator[](int i) { return p[i]; }
+    __device__ __forceinline__ T *ptr() { return p; }
+};
+
+// A team-level globalized variable allocated by the main thread only and read
+// by the team's threads inside parallel regions.
+//   generic, RUNTIME/GLOBAL : main allocates on its stack; pointer passed
+//   generic, SHARED_STATIC  : static __shared__ (heap-to-shared)
+//   generic, STACK          : heap-to-stack is illegal (the pointer escapes to
+//                             the workers) -> heap-to-shared, as h2s2 does
+//   SPMD,    STACK          : every thread owns a copy (no escape once the
+//                             region runs in place); writes need no guard
+//   SPMD,    SHARED_STATIC  : one shared copy; writes guarded by thread 0
+//   SPMD,    RUNTIME/GLOBAL : thread 0 allocates, pointer broadcast; writes
+//                             guarded
+//
+// RO = the parallel regions only read it.  If they write it (the variable is
+// shared between the team's threads, e.g. Fig. 1's team_val), SPMD + STACK
+// cannot privatize it and uses static shared memory instead.
+template <class K, class T, class Tag, bool RO = true> struct TeamLocal {
+    static constexpr bool PRIVATE = (K::MODE == SPMD && K::PL == PL_STACK && RO);
+    static constexpr bool RUNTIME_ALLOC = (K::PL == PL_RUNTIME || K::PL == PL_GLOBAL);
+    T priv;
+    T *p;
+    __device__ __forceinline__ static T *static_slot() {
+        __shared__ T s;
+        return &s;
+    }
+    __device__ __forceinline__ TeamLocal() {
+        if constexpr (PRIVATE) {
+            p = &priv;
+        } else if constexpr (RUNTIME_ALLOC) {
+            if constexpr (K::MODE == SPMD)
+                p = guarded_bcast<K, T *>([] { return static_cast<T *>(alloc_shared<K>(sizeof(T))); });
+            else
+                p = static_cast<T *>(alloc_shared<K>(sizeof(T)));
+        } else {
+            p = static_slot();
+        }
+    }
+    __device__ __forceinline__ ~TeamLocal() {
+        if constexpr (RUNTIME_ALLOC) {
+            if constexpr (K::MODE == SPMD) {
+                __syncthreads();
+                if (threadIdx.x == 0) free_shared<K>(p, sizeof(T));
+            } else {
+                free_shared<K>(p, sizeof(T));
+            }
+        }
+    }
+    // write by "the main thread": guarded in SPMD unless private
+    template <class F> __device__ __forceinline__ void set(F &&f) {
+        if constexpr (PRIVATE || K::MODE != SPMD) f(*p);
+        else guarded<K>([&] { f(*p); });
+    }
+    __device__ __forceinline__ T *get() { return p; }
+};
+
+// ---------------------------------------------------------------- worksharing
+// `for` with a static schedule, chunk 1 (cyclic) -- AMB-2: coalesced.
+template <class K, class F> __device__ __forceinline__ void for_static(int64_t lo, int64_t hi, F &&body) {
+    const int64_t t = thread_num<K>(), n = num_threads<K>();
+    for (int64_t i = lo + t; i < hi; i += n) body(i);
+}
+
+// ---------------------------------------------------------------- reductions
+// Team reduction of small integer tallies: shared-memory atomics per event,
+// one global atomic per counter per team at the end.
+__device__ __forceinline__ void tally_flush(const uint32_t *s, int n, unsigned long long *g, int tid, int nthr) {
+    for (int k = tid; k < n; k += nthr)
+        if (s[k]) atomicAdd(&g[k], (unsigned long long)s[k]);
+}
+
+}  // namespace gtr

@@ -1,0 +1,97 @@
+// rs.cu -- RS lookup entry points: variant dispatch, the NATIVE (CUDA
+// watermark) kernel and the extern "C" API.
+#include "rs_impl.cuh"
+
+namespace gtr {
+namespace rs {
+
+template <class K> int run_variant(LaunchArgs &a);
+template <class K> struct VariantOp {
+    static int run(LaunchArgs &a) { return run_variant<K>(a); }
+};
+
+template <int NT> __global__ void __launch_bounds__(NT) kernel_native(Params P) {
+    using KN = Cfg<NATIVE, PL_STACK, true, NT>;
+    __shared__ uint32_t tally[17];
+    if (threadIdx.x < 17) tally[threadIdx.x] = 0;
+    __syncthreads();
+    const uint64_t stride = (uint64_t)gridDim.x * NT;
+    for (uint64_t k = (uint64_t)blockIdx.x * NT + threadIdx.x; k < P.n; k += stride)
+        lookup<KN>(P, P.first + k, tally);
+    __syncthreads();
+    flush(tally, P.out, threadIdx.x, NT);
+}
+
+template <int NT> int run_native(LaunchArgs &a) {
+    const void *fn = reinterpret_cast<const void *>(&kernel_native<NT>);
+    int per_sm = 0;
+    GTR_CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, fn, NT, 0));
+    Launch L;
+    L.block = NT;
+    L.dyn_smem = 0;
+    L.teams = a.cfg->num_teams > 0 ? a.cfg->num_teams : per_sm * a.ctx->num_sms;
+    if (a.info) return fill_info<Cfg<NATIVE, PL_STACK, true, NT>>(fn, L, per_sm, a.info);
+    kernel_native<NT><<<L.teams, NT, 0, a.stream>>>(a.P);
+    GTR_CUDA_TRY(cudaGetLastError());
+    return GTR_OK;
+}
+
+inline int launch(LaunchArgs &a) {
+    const gtr_launch_cfg *c = a.cfg;
+    if (!valid_cfg(c)) return GTR_EINVAL;
+    if (c->mode == NATIVE) {
+        if (c->thread_limit == 128) return run_native<128>(a);
+        if (c->thread_limit == 256) return run_native<256>(a);
+        return GTR_EUNSUPPORTED;
+    }
+    if (c->thread_limit == 128) return dispatch_mpf<128, 0, VariantOp>(c->mode, c->placement, c->fold, a);
+    return GTR_EUNSUPPORTED;
+}
+
+}  // namespace rs
+}  // namespace gtr
+
+using namespace gtr;
+
+static rs::Params make_params(const gtr_rs_tables *t, uint64_t first, uint64_t n, uint64_t seed,
+                              uint64_t *d_out, const gtr_rs_verify *v) {
+    rs::Params P{};
+    if (t) {
+        P.n_windows = t->n_windows;
+        P.poles = t->poles;
+        P.windows = t->windows;
+        P.k0rs = t->k0rs;
+        P.num_nucs = t->num_nucs;
+        P.mats = t->mats;
+        P.concs = t->concs;
+        P.n_nuc = t->n_nuc;
+        P.max_poles = t->max_poles;
+        P.max_windows = t->max_windows;
+        P.max_num_nucs = t->max_num_nucs;
+    }
+    P.first = first;
+    P.n = n;
+    P.seed = seed;
+    P.v_mat = v ? v->mat : nullptr;
+    P.v_am = v ? v->am : nullptr;
+    P.v_macro = v ? v->macro : nullptr;
+    P.out = reinterpret_cast<unsigned long long *>(d_out);
+    return P;
+}
+
+int gtr_internal_query_rs(gtr_ctx *ctx, const gtr_launch_cfg *cfg, gtr_variant_info *info) {
+    rs::LaunchArgs a{ctx, cfg, make_params(nullptr, 0, 0, 0, nullptr, nullptr), nullptr, info};
+    return rs::launch(a);
+}
+
+extern "C" int gtr_rs_lookup(gtr_ctx *ctx, const gtr_launch_cfg *cfg, const gtr_rs_tables *t, uint64_t first,
+                             uint64_t n, uint64_t seed, uint64_t *d_out, const gtr_rs_verify *verify,
+                             void *stream) {
+    if (!ctx || !cfg || !t || !d_out || !t->n_windows || !t->poles || !t->windows || !t->k0rs ||
+        !t->num_nucs || !t->mats || !t->concs || t->n_nuc < 1 || t->max_poles < 1 || t->max_windows < 1)
+        return GTR_EINVAL;
+    if (n == 0) return GTR_OK;
+    rs::LaunchArgs a{ctx, cfg, make_params(t, first, n, seed, d_out, verify), static_cast<cudaStream_t>(stream),
+                     nullptr};
+    return rs::launch(a);
+}

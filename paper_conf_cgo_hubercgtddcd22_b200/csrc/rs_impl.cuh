@@ -1,0 +1,279 @@
+// rs_impl.cuh -- RSBench-style windowed multipole cross-section lookup
+// (BASELINE config 4) on the team runtime.
+//
+// Paper: RSBench is the compute-bound alternative to XSBench,
+// timed as `rsbench -s large -m event`; already SPMD, 7 globalized
+// variables (Fig. 9) whose runtime globalization caused OOM or
+// "tremendous slowdowns" until heap-to-stack applied.
+// Algorithm step by step as in oracle/rs.c (R1-R6),
+// written independently here.  Globalized per-lookup variables (AMB-7):
+// seed, macro[4], micro[4], sigTfactors[4] (complex), Z, W, sig[3].
+// Shapes as XS: GENERIC/CASCADE/CSM `teams distribute` over lookup chunks with
+// a forked `parallel for`; SPMD-ized; NATIVE thread per lookup.
+#pragma once
+#include <cfloat>
+
+#include "gtr_internal.h"
+#include "sampling.cuh"
+
+namespace gtr {
+namespace rs {
+
+struct Params {
+    const int32_t *n_windows;
+    const double *poles;      // 9 words per record
+    const double *windows;    // 4 words per record
+    const double *k0rs;
+    const int32_t *num_nucs;
+    const int32_t *mats;
+    const double *concs;
+    int64_t n_nuc, max_poles, max_windows;
+    int32_t max_num_nucs;
+    uint32_t chunk;
+    uint64_t first, n, seed;
+    uint8_t *v_mat;
+    uint8_t *v_am;
+    double *v_macro;
+    unsigned long long *out;
+};
+
+// ---- complex arithmetic in RSBench's operation order ----------------------
+struct cx {
+    double r, i;
+};
+__device__ __forceinline__ cx cadd(cx a, cx b) { return {a.r + b.r, a.i + b.i}; }
+__device__ __forceinline__ cx csub(cx a, cx b) { return {a.r - b.r, a.i - b.i}; }
+__device__ __forceinline__ cx cmul(cx a, cx b) { return {a.r * b.r - a.i * b.i, a.r * b.i + a.i * b.r}; }
+__device__ __forceinline__ cx cdiv(cx a, cx b) {
+    const double d = b.r * b.r + b.i * b.i;
+    return {((a.r * b.r) + (a.i * b.i)) / d, ((a.i * b.r) - (a.r * b.i)) / d};
+}
+__device__ __forceinline__ double cabs_(cx a) { return sqrt(a.r * a.r + a.i * a.i); }
+
+__device__ __forceinline__ double fast_exp(double x) {
+    x = 1.0 + x * 0.000244140625;
+#pragma unroll
+    for (int k = 0; k < 12; k++) x *= x;
+    return x;
+}
+__device__ __forceinline__ cx fast_cexp(cx z) {
+    const double t1 = fast_exp(z.r);
+    double s, c;
+    sincos(z.i, &s, &c);
+    return {t1 * c, t1 * s};
+}
+
+// Faddeeva W(z): Abrarov series (N = 10, Tm = 12) inside |z| < 6, two-pole
+// asymptotic expansion outside; RSBench's tabulated constants.
+__device__ __forceinline__ cx faddeeva(cx Z) {
+    if (cabs_(Z) < 6.0) {
+        const double an[10] = {2.758402e-01, 2.245740e-01, 1.594149e-01, 9.866577e-02, 5.324414e-02,
+                               2.505215e-02, 1.027747e-02, 3.676164e-03, 1.146494e-03, 3.117570e-04};
+        const double dl[10] = {9.869604e+00, 3.947842e+01, 8.882644e+01, 1.579137e+02, 2.467401e+02,
+                               3.553058e+02, 4.836106e+02, 6.316547e+02, 7.994379e+02, 9.869604e+02};
+        const cx prefactor = {0.0, 8.124330e+01};
+        const cx t1 = {0.0, 12.0}, t2 = {12.0, 0.0}, I = {0.0, 1.0}, one = {1.0, 0.0};
+        const cx e12 = fast_cexp(cmul(t1, Z));
+        cx W = cdiv(cmul(I, csub(one, e12)), cmul(t2, Z));
+        cx sum = {0.0, 0.0};
+#pragma unroll
+        for (int n = 0; n < 10; n++) {
+            const cx t3 = {(n & 1) ? 1.0 : -1.0, 0.0};
+            const cx top = csub(cmul(t3, e12), one);
+            const cx t4 = {dl[n], 0.0}, t5 = {144.0, 0.0};
+            const cx bot = csub(t4, cmul(t5, cmul(Z, Z)));
+            const cx t6 = {an[n], 0.0};
+            sum = cadd(sum, cmul(t6, cdiv(top, bot)));
+        }
+        return cadd(W, cmul(prefactor, cmul(Z, sum)));
+    }
+    const cx a = {0.512424224754768462984202823134979415014943561548661637413182, 0.0};
+    const cx b = {0.275255128608410950901357962647054304017026259671664935783653, 0.0};
+    const cx c = {0.051765358792987823963876628425793170829107067780337219430904, 0.0};
+    const cx d = {2.724744871391589049098642037352945695982973740328335064216346, 0.0};
+    const cx I = {0.0, 1.0};
+    const cx Z2 = cmul(Z, Z);
+    return cmul(cmul(Z, I), cadd(cdiv(a, csub(Z2, b)), cdiv(c, csub(Z2, d))));
+}
+
+struct TagSeed {};
+struct TagMacro {};
+struct TagMicro {};
+struct TagSigTF {};
+struct TagZ {};
+struct TagW {};
+struct TagSig {};
+
+// microscopic XS of nuclide nuc at energy E (4 channels) into micro
+template <class K, class LM>
+__device__ __forceinline__ void micro_xs(const Params &P, int64_t nuc, double E, LM &micro) {
+    Local<K, double, 8, TagSigTF> sf;     // sigTfactors[4] complex
+    Local<K, double, 2, TagZ> Zv;
+    Local<K, double, 2, TagW> Wv;
+    Local<K, double, 3, TagSig> sig;
+    const int32_t nw = __ldg(P.n_windows + nuc);
+    const double spacing = 1.0 / nw;
+    int32_t window = (int32_t)(E / spacing);
+    if (window == nw) window--;
+    const double sqE = sqrt(E);
+#pragma unroll
+    for (int l = 0; l < 4; l++) {
+        double phi = __ldg(P.k0rs + nuc * 4 + l) * sqE;
+        if (l == 1) phi -= -atan(phi);
+        else if (l == 2) phi -= atan(3.0 * phi / (3.0 - phi * phi));
+        else if (l == 3) phi -= atan(phi * (15.0 - phi * phi) / (15.0 - 6.0 * phi * phi));
+        phi *= 2.0;
+        double s, c;
+        sincos(phi, &s, &c);
+        sf[2 * l] = c;
+        sf[2 * l + 1] = -s;
+    }
+    const double *w = P.windows + (nuc * P.max_windows + window) * 4;
+    const int2 se = *reinterpret_cast<const int2 *>(w + 3);
+    sig[0] = E * __ldg(w + 0);
+    sig[1] = E * __ldg(w + 1);
+    sig[2] = E * __ldg(w + 2);
+    for (int32_t p = se.x; p < se.y; p++) {
+        const double *pr = P.poles + (nuc * P.max_poles + p) * 9;
+        // 72-byte records: 8-byte aligned only, so scalar loads
+        const double2 EA = make_double2(__ldg(pr + 0), __ldg(pr + 1));
+        const double2 RT = make_double2(__ldg(pr + 2), __ldg(pr + 3));
+        const double2 RA = make_double2(__ldg(pr + 4), __ldg(pr + 5));
+        const double2 RF = make_double2(__ldg(pr + 6), __ldg(pr + 7));
+        const int lv = __ldg(reinterpret_cast<const int *>(pr + 8));
+        const cx Z = cmul(csub(cx{E, 0.0}, cx{EA.x, EA.y}), cx{0.5, 0.0});
+        Zv[0] = Z.r;
+        Zv[1] = Z.i;
+        const cx W = faddeeva(cx{Zv[0], Zv[1]});
+        Wv[0] = W.r;
+        Wv[1] = W.i;
+        const cx Wl = {Wv[0], Wv[1]};
+        const cx f = {sf[2 * lv], sf[2 * lv + 1]};
+        sig[0] = sig[0] + cmul(cx{RT.x, RT.y}, cmul(Wl, f)).r;
+        sig[1] = sig[1] + cmul(cx{RA.x, RA.y}, Wl).r;
+        sig[2] = sig[2] + cmul(cx{RF.x, RF.y}, Wl).r;
+    }
+    micro[0] = sig[0];
+    micro[1] = sig[1];
+    micro[2] = sig[2];
+    micro[3] = sig[0] - sig[1];
+}
+
+template <class K>
+__device__ __forceinline__ void lookup(const Params &P, uint64_t i, uint32_t *tally) {
+    Local<K, uint64_t, 1, TagSeed> seed;
+    Local<K, double, 4, TagMacro> macro;
+    Local<K, double, 4, TagMicro> micro;
+    seed[0] = smp::lcg_jump(P.seed, 2ULL * i);
+    const double E = smp::lcg_uniform(seed[0]);
+    const int mat = smp::sample_material(seed[0]);
+#pragma unroll
+    for (int c = 0; c < 4; c++) macro[c] = 0.0;
+    const int nn = __ldg(P.num_nucs + mat);
+    for (int j = 0; j < nn; j++) {
+        const int64_t nuc = __ldg(P.mats + (int64_t)mat * P.max_num_nucs + j);
+        const double conc = __ldg(P.concs + (int64_t)mat * P.max_num_nucs + j);
+        micro_xs<K>(P, nuc, E, micro);
+#pragma unroll
+        for (int c = 0; c < 4; c++) macro[c] += micro[c] * conc;
+    }
+    double mx = -DBL_MAX;
+    int am = 0;
+#pragma unroll
+    for (int c = 0; c < 4; c++)
+        if (macro[c] > mx) { mx = macro[c]; am = c; }
+    atomicAdd(&tally[mat], 1u);
+    atomicAdd(&tally[12 + am], 1u);
+    const uint64_t o = i - P.first;
+    if (P.v_mat) P.v_mat[o] = (uint8_t)mat;
+    if (P.v_am) P.v_am[o] = (uint8_t)am;
+    if (P.v_macro) {
+#pragma unroll
+        for (int c = 0; c < 4; c++) P.v_macro[o * 4 + c] = macro[c];
+    }
+}
+
+__device__ __forceinline__ void flush(const uint32_t *tally, unsigned long long *out, int tid, int nthr) {
+    if (tid == 0) {
+        unsigned long long h = 0;
+        for (int a = 0; a < 4; a++) h += (unsigned long long)(a + 1) * tally[12 + a];
+        if (h) atomicAdd(&out[0], h);
+    }
+    for (int k = tid; k < 17; k += nthr)
+        if (tally[k]) atomicAdd(&out[1 + k], (unsigned long long)tally[k]);
+}
+
+static __shared__ Params g_p;
+static __shared__ uint32_t g_tally[17];
+
+struct Chunk {
+    uint64_t base, count;
+};
+struct TagChunk {};
+
+template <class K> struct LookupRegion {
+    static constexpr int ID = 1;
+    static __device__ void run(void *a) {
+        const Chunk *c = static_cast<const Chunk *>(a);
+        const uint64_t base = c->base, cnt = c->count;
+        for_static<K>(0, (int64_t)cnt, [&](int64_t k) { lookup<K>(g_p, base + (uint64_t)k, g_tally); });
+    }
+};
+
+template <class K> __global__ void __launch_bounds__(K::BLOCK) kernel_rt(Params P, RtParams rp) {
+    const Role role = team_init<K>(rp);
+    if (role == Role::Exit) return;
+    if (role == Role::Worker) {
+        worker_loop<K, LookupRegion<K>>();
+        return;
+    }
+    guarded<K>([&] {
+        g_p = P;
+        for (int k = 0; k < 17; k++) g_tally[k] = 0;
+    });
+    const uint64_t n = P.n, ch = P.chunk;
+    const uint64_t nchunks = (n + ch - 1) / ch;
+    for (uint64_t c = team_num<K>(); c < nchunks; c += num_teams<K>()) {
+        TeamLocal<K, Chunk, TagChunk> chunk;
+        chunk.set([&](Chunk &x) {
+            x.base = P.first + c * ch;
+            x.count = (c * ch + ch <= n) ? ch : n - c * ch;
+        });
+        parallel<K, LookupRegion<K>>(chunk.get());
+    }
+    if constexpr (K::MODE == SPMD) flush(g_tally, g_p.out, threadIdx.x, K::NT);
+    else flush(g_tally, g_p.out, 0, 1);
+    team_deinit<K>();
+}
+
+struct LaunchArgs {
+    gtr_ctx *ctx;
+    const gtr_launch_cfg *cfg;
+    Params P;
+    cudaStream_t stream;
+    gtr_variant_info *info;
+};
+
+constexpr uint32_t kDefaultStackBytes = 256;   // 192 B per-lookup locals + chunk
+constexpr uint32_t kLookupsPerThreadPerChunk = 2;
+
+template <class K> struct OpRt {
+    static int run(LaunchArgs &a) {
+        const void *fn = reinterpret_cast<const void *>(&kernel_rt<K>);
+        Launch L;
+        int st = resolve<K>(a.ctx, a.cfg, fn, kDefaultStackBytes, &L);
+        if (st) return st;
+        if (a.info) {
+            int per_sm = 0;
+            GTR_CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, fn, K::BLOCK, L.dyn_smem));
+            return fill_info<K>(fn, L, per_sm, a.info);
+        }
+        a.P.chunk = kLookupsPerThreadPerChunk * K::NT;
+        kernel_rt<K><<<L.teams, L.block, L.dyn_smem, a.stream>>>(a.P, L.rp);
+        GTR_CUDA_TRY(cudaGetLastError());
+        return GTR_OK;
+    }
+};
+
+}  // namespace rs
+}  // namespace gtr

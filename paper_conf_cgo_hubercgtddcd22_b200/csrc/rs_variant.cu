@@ -1,0 +1,12 @@
+// rs_variant.cu -- one module per runtime-mode variant of the RS lookup
+// (see xs_variant.cu and build.py).
+#include "rs_impl.cuh"
+#include "variant_inst.h"
+
+namespace gtr {
+namespace rs {
+template <class K> int run_variant(LaunchArgs &a) { return OpRt<K>::run(a); }
+#define GTR_INST(M, P, F, NT, FL) template int run_variant<Cfg<M, P, F, NT, FL>>(LaunchArgs &);
+GTR_VARIANT_INSTANCES
+}  // namespace rs
+}  // namespace gtr

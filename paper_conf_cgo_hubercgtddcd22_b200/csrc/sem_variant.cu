@@ -1,0 +1,12 @@
+// sem_variant.cu -- one module per runtime-mode variant of the semantic
+// programs (see xs_variant.cu and build.py).
+#include "sem_impl.cuh"
+#include "variant_inst.h"
+
+namespace gtr {
+namespace sem {
+template <class K> int run_variant(LaunchArgs &a) { return OpRt<K>::run(a); }
+#define GTR_INST(M, P, F, NT, FL) template int run_variant<Cfg<M, P, F, NT, FL>>(LaunchArgs &);
+GTR_VARIANT_INSTANCES
+}  // namespace sem
+}  // namespace gtr

@@ -1,0 +1,200 @@
+// xs.cu -- XS entry points: variant dispatch, the NATIVE (CUDA watermark)
+// kernel, the unionized-grid builders and the extern "C" API (include/gtr.h).
+// The runtime-mode variants live in separate modules (xs_variant.cu compiled
+// once per variant): a GENERIC kernel's indirect
+// call may reach every address-taken region of its module, so sharing a
+// module across variants would inflate each one's registers and shared
+// memory (the spurious call edges of P:593-597, fn. 4).
+#include "xs_impl.cuh"
+
+namespace gtr {
+namespace xs {
+
+// ---------------------------------------------------------------- native form
+template <int NT> __global__ void __launch_bounds__(NT) kernel_native(Params P) {
+    using KN = Cfg<NATIVE, PL_STACK, true, NT>;
+    __shared__ uint32_t tally[17];
+    if (threadIdx.x < 17) tally[threadIdx.x] = 0;
+    if (P.req) { P.first = P.req->first; P.n = P.req->n; P.seed = P.req->seed; }
+    __syncthreads();
+    const uint64_t stride = (uint64_t)gridDim.x * NT;
+    for (uint64_t k = (uint64_t)blockIdx.x * NT + threadIdx.x; k < P.n; k += stride)
+        lookup<KN>(P, P.first + k, tally);
+    __syncthreads();
+    flush(tally, P.out, threadIdx.x, NT);
+}
+
+// ---------------------------------------------------------------- builders
+// energies e[n][k] = grid[n][k][0]
+__global__ void k_extract_energies(const double *__restrict__ grid, int64_t total, double *__restrict__ e) {
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < total;
+         i += (int64_t)gridDim.x * blockDim.x)
+        e[i] = __ldg(grid + i * 6);
+}
+// number of entries of sorted a[0..n) that are < x (strict) or <= x
+__device__ __forceinline__ int64_t count_below(const double *__restrict__ a, int64_t n, double x, bool inclusive) {
+    int64_t lo = 0, hi = n;   // answer in [lo, hi]
+    while (lo < hi) {
+        int64_t mid = (lo + hi) >> 1;
+        double v = __ldg(a + mid);
+        if (inclusive ? (v <= x) : (v < x)) lo = mid + 1;
+        else hi = mid;
+    }
+    return lo;
+}
+// position of energy (n,k) in the union = number of smaller energies
+__global__ void k_union_scatter(const double *__restrict__ e, int64_t n_iso, int64_t n_gp,
+                                double *__restrict__ egrid) {
+    const int64_t total = n_iso * n_gp;
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < total;
+         i += (int64_t)gridDim.x * blockDim.x) {
+        const double x = e[i];
+        int64_t rank = 0;
+        for (int64_t m = 0; m < n_iso; m++) rank += count_below(e + m * n_gp, n_gp, x, false);
+        egrid[rank] = x;
+    }
+}
+__global__ void k_fill_nan(double *p, int64_t n) {
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+        p[i] = __longlong_as_double(0x7FF8000000000000LL);
+}
+// strictly increasing (also catches unwritten NaN slots = duplicate ranks)
+__global__ void k_check_increasing(const double *__restrict__ eg, int64_t n, uint32_t *err) {
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n;
+         i += (int64_t)gridDim.x * blockDim.x) {
+        const double a = eg[i];
+        bool ok = (a == a);
+        if (i + 1 < n) ok = ok && (eg[i + 1] > a);
+        if (!ok) atomicOr(err, (uint32_t)ERR_DUP_ENERGY);
+    }
+}
+// index[u][n] = clamp(#{k: e_n[k] <= egrid[u]} - 1, 0, n_gp - 2)
+__global__ void k_index_grid(const double *__restrict__ e, int64_t n_iso, int64_t n_gp,
+                             const double *__restrict__ egrid, int64_t n_union, int32_t *__restrict__ idx) {
+    const int64_t total = n_union * n_iso;
+    for (int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; t < total;
+         t += (int64_t)gridDim.x * blockDim.x) {
+        const int64_t u = t / n_iso, n = t - u * n_iso;
+        int64_t c = count_below(e + n * n_gp, n_gp, __ldg(egrid + u), true) - 1;
+        c = c < 0 ? 0 : (c > n_gp - 2 ? n_gp - 2 : c);
+        idx[t] = (int32_t)c;
+    }
+}
+
+// Runtime-mode variants: defined (explicitly instantiated) in xs_variant.cu.
+template <class K> int run_variant(LaunchArgs &a);
+template <class K> struct VariantOp {
+    static int run(LaunchArgs &a) { return run_variant<K>(a); }
+};
+
+template <int NT> int run_native(LaunchArgs &a) {
+    const void *fn = reinterpret_cast<const void *>(&kernel_native<NT>);
+    int per_sm = 0;
+    GTR_CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, fn, NT, 0));
+    Launch L;
+    L.block = NT;
+    L.dyn_smem = 0;
+    L.teams = a.cfg->num_teams > 0 ? a.cfg->num_teams : per_sm * a.ctx->num_sms;
+    if (a.info) return fill_info<Cfg<NATIVE, PL_STACK, true, NT>>(fn, L, per_sm, a.info);
+    kernel_native<NT><<<L.teams, NT, 0, a.stream>>>(a.P);
+    GTR_CUDA_TRY(cudaGetLastError());
+    return GTR_OK;
+}
+
+inline int launch(LaunchArgs &a) {
+    const gtr_launch_cfg *c = a.cfg;
+    if (!valid_cfg(c)) return GTR_EINVAL;
+    if (c->mode == NATIVE) {
+        if (c->thread_limit == 128) return run_native<128>(a);
+        if (c->thread_limit == 256) return run_native<256>(a);
+        if (c->thread_limit == 512) return run_native<512>(a);
+        return GTR_EUNSUPPORTED;
+    }
+    if (c->thread_limit == 128) return dispatch_mpf<128, 0, VariantOp>(c->mode, c->placement, c->fold, a);
+    if (c->thread_limit == 256) return dispatch_mpf<256, 0, VariantOp>(c->mode, c->placement, c->fold, a);
+    return GTR_EUNSUPPORTED;
+}
+
+}  // namespace xs
+}  // namespace gtr
+
+using namespace gtr;
+
+int gtr_internal_query_xs(gtr_ctx *ctx, const gtr_launch_cfg *cfg, gtr_variant_info *info) {
+    gtr_xs_tables t = {};
+    xs::LaunchArgs a{ctx, cfg, xs::make_params(&t, 0, 0, 0, nullptr, nullptr, nullptr), nullptr, info};
+    return xs::launch(a);
+}
+
+extern "C" uint64_t gtr_xs_build_workspace_bytes(int64_t n_iso, int64_t n_gp) {
+    return (uint64_t)n_iso * (uint64_t)n_gp * 8u;
+}
+
+static int grid_blocks(gtr_ctx *ctx, int64_t work, int threads) {
+    int64_t b = (work + threads - 1) / threads;
+    int64_t cap = (int64_t)ctx->num_sms * 16;
+    return (int)(b < 1 ? 1 : (b > cap ? cap : b));
+}
+
+extern "C" int gtr_xs_build_egrid(gtr_ctx *ctx, const double *d_grid, int64_t n_iso, int64_t n_gp,
+                                  double *d_egrid_out, void *d_workspace, void *stream) {
+    if (!ctx || !d_grid || !d_egrid_out || !d_workspace || n_iso < 1 || n_gp < 2) return GTR_EINVAL;
+    cudaStream_t s = static_cast<cudaStream_t>(stream);
+    const int64_t total = n_iso * n_gp;
+    double *e = static_cast<double *>(d_workspace);
+    xs::k_extract_energies<<<grid_blocks(ctx, total, 256), 256, 0, s>>>(d_grid, total, e);
+    xs::k_fill_nan<<<grid_blocks(ctx, total, 256), 256, 0, s>>>(d_egrid_out, total);
+    xs::k_union_scatter<<<grid_blocks(ctx, total, 128), 128, 0, s>>>(e, n_iso, n_gp, d_egrid_out);
+    xs::k_check_increasing<<<grid_blocks(ctx, total, 256), 256, 0, s>>>(d_egrid_out, total, ctx->d_err);
+    GTR_CUDA_TRY(cudaGetLastError());
+    return GTR_OK;
+}
+
+extern "C" int gtr_xs_build_index_grid(gtr_ctx *ctx, const double *d_grid, int64_t n_iso, int64_t n_gp,
+                                       const double *d_egrid, int32_t *d_index_out, void *d_workspace,
+                                       void *stream) {
+    if (!ctx || !d_grid || !d_egrid || !d_index_out || !d_workspace || n_iso < 1 || n_gp < 2)
+        return GTR_EINVAL;
+    cudaStream_t s = static_cast<cudaStream_t>(stream);
+    const int64_t total = n_iso * n_gp;
+    double *e = static_cast<double *>(d_workspace);
+    xs::k_extract_energies<<<grid_blocks(ctx, total, 256), 256, 0, s>>>(d_grid, total, e);
+    xs::k_index_grid<<<grid_blocks(ctx, total * n_iso, 256), 256, 0, s>>>(e, n_iso, n_gp, d_egrid, total,
+                                                                          d_index_out);
+    GTR_CUDA_TRY(cudaGetLastError());
+    return GTR_OK;
+}
+
+static bool tables_ok(const gtr_xs_tables *t) {
+    return t && t->egrid && t->index_grid && t->grid && t->num_nucs && t->mats && t->concs &&
+           t->n_iso > 0 && t->n_gp >= 2 && t->n_union >= 2 && t->n_union < (int64_t)UINT32_MAX &&
+           t->max_num_nucs > 0;
+}
+
+extern "C" int gtr_xs_lookup(gtr_ctx *ctx, const gtr_launch_cfg *cfg, const gtr_xs_tables *tables,
+                             uint64_t first, uint64_t n, uint64_t seed, uint64_t *d_out,
+                             const gtr_xs_verify *verify, void *stream) {
+    if (!ctx || !cfg || !tables_ok(tables) || !d_out) return GTR_EINVAL;
+    if (n == 0) return GTR_OK;
+    xs::LaunchArgs a{ctx, cfg, xs::make_params(tables, first, n, seed, d_out, verify, nullptr),
+                     static_cast<cudaStream_t>(stream), nullptr};
+    return xs::launch(a);
+}
+
+extern "C" int gtr_xs_lookup_host(gtr_ctx *ctx, const gtr_launch_cfg *cfg, const gtr_xs_tables *tables,
+                                  const gtr_xs_request *h_req, uint64_t *h_out, void *stream) {
+    if (!ctx || !cfg || !tables_ok(tables) || !h_req || !h_out) return GTR_EINVAL;
+    cudaStream_t s = static_cast<cudaStream_t>(stream);
+    gtr_xs_request *d_req = static_cast<gtr_xs_request *>(ctx->d_stage);
+    uint64_t *d_out = reinterpret_cast<uint64_t *>(static_cast<char *>(ctx->d_stage) + 64);
+    GTR_CUDA_TRY(cudaMemcpyAsync(d_req, h_req, sizeof(gtr_xs_request), cudaMemcpyHostToDevice, s));
+    GTR_CUDA_TRY(cudaMemsetAsync(d_out, 0, 18 * sizeof(uint64_t), s));
+    // the kernel reads (first, n, seed) from d_req; n bounds the launch only
+    xs::LaunchArgs a{ctx, cfg, xs::make_params(tables, h_req->first, h_req->n, h_req->seed, d_out, nullptr, d_req),
+                     s, nullptr};
+    int st = xs::launch(a);
+    if (st) return st;
+    GTR_CUDA_TRY(cudaMemcpyAsync(h_out, d_out, 18 * sizeof(uint64_t), cudaMemcpyDeviceToHost, s));
+    GTR_CUDA_TRY(cudaStreamSynchronize(s));
+    return GTR_OK;
+}

@@ -1,0 +1,78 @@
+"""Device-resident problems: upload the generator's tables with PyTorch (device
+memory only) and build the XS acceleration structures with libgtr's own
+kernels.  Plumbing -- no arithmetic of the method happens in Python.
+"""
+import numpy as np
+import torch
+
+from . import gtr as G
+
+
+def _dev(a, device):
+    return torch.from_numpy(np.ascontiguousarray(a)).to(device, non_blocking=False)
+
+
+class XsDevice:
+    """XS tables on the GPU: the nuclide grid (uploaded), the unionized energy
+    grid and the index grid (built by gtr_xs_build_egrid / _index_grid)."""
+
+    def __init__(self, ctx, t, device="cuda", stream=None):
+        self.n_iso, self.n_gp = int(t["n_iso"]), int(t["n_gp"])
+        self.n_union = self.n_iso * self.n_gp
+        self.grid = _dev(t["grid"], device)
+        self.num_nucs = _dev(t["num_nucs"].astype(np.int32), device)
+        self.mats = _dev(t["mats"].astype(np.int32), device)
+        self.concs = _dev(t["concs"].astype(np.float64), device)
+        self.max_num_nucs = int(t["mats"].shape[1])
+        self.egrid = torch.empty(self.n_union, dtype=torch.float64, device=device)
+        self.index_grid = torch.empty((self.n_union, self.n_iso), dtype=torch.int32, device=device)
+        ws = torch.empty(G.gtr_xs_build_workspace_bytes(self.n_iso, self.n_gp), dtype=torch.uint8, device=device)
+        G.gtr_xs_build_egrid(ctx, self.grid, self.n_iso, self.n_gp, self.egrid, ws, stream)
+        G.gtr_xs_build_index_grid(ctx, self.grid, self.n_iso, self.n_gp, self.egrid, self.index_grid, ws, stream)
+        G.gtr_ctx_check(ctx, stream)           # duplicate energies -> GtrError
+        del ws
+        self.tables = G.gtr_xs_tables(self.n_iso, self.n_gp, self.n_union, self.max_num_nucs,
+                                      self.egrid.data_ptr(), self.index_grid.data_ptr(), self.grid.data_ptr(),
+                                      self.num_nucs.data_ptr(), self.mats.data_ptr(), self.concs.data_ptr())
+
+    def nbytes(self):
+        return sum(x.numel() * x.element_size() for x in
+                   (self.grid, self.egrid, self.index_grid, self.num_nucs, self.mats, self.concs))
+
+    def verify_buffers(self, n, device="cuda"):
+        bufs = {"mat": torch.zeros(n, dtype=torch.uint8, device=device),
+                "u": torch.zeros(n, dtype=torch.int32, device=device),
+                "am": torch.zeros(n, dtype=torch.uint8, device=device),
+                "macro": torch.zeros((n, 5), dtype=torch.float64, device=device)}
+        v = G.gtr_xs_verify(bufs["mat"].data_ptr(), bufs["u"].data_ptr(), bufs["am"].data_ptr(),
+                            bufs["macro"].data_ptr())
+        return v, bufs
+
+
+class RsDevice:
+    def __init__(self, t, device="cuda"):
+        self.n_windows = _dev(t["n_windows"].astype(np.int32), device)
+        self.poles = _dev(np.ascontiguousarray(t["poles"]).view(np.uint8), device)
+        self.windows = _dev(np.ascontiguousarray(t["windows"]).view(np.uint8), device)
+        self.k0rs = _dev(t["k0rs"].astype(np.float64), device)
+        self.num_nucs = _dev(t["num_nucs"].astype(np.int32), device)
+        self.mats = _dev(t["mats"].astype(np.int32), device)
+        self.concs = _dev(t["concs"].astype(np.float64), device)
+        self.tables = G.gtr_rs_tables(int(t["n_nuc"]), int(t["max_poles"]), int(t["max_windows"]),
+                                      int(t["mats"].shape[1]), self.n_windows.data_ptr(), self.poles.data_ptr(),
+                                      self.windows.data_ptr(), self.k0rs.data_ptr(), self.num_nucs.data_ptr(),
+                                      self.mats.data_ptr(), self.concs.data_ptr())
+
+    def verify_buffers(self, n, device="cuda"):
+        bufs = {"mat": torch.zeros(n, dtype=torch.uint8, device=device),
+                "am": torch.zeros(n, dtype=torch.uint8, device=device),
+                "macro": torch.zeros((n, 4), dtype=torch.float64, device=device)}
+        v = G.gtr_rs_verify(bufs["mat"].data_ptr(), bufs["am"].data_ptr(), bufs["macro"].data_ptr())
+        return v, bufs
+
+
+def su3_device(A, B, device="cuda"):
+    """complex128 numpy arrays -> float64 device tensors [..., 2] (same bytes)."""
+    dA = _dev(np.ascontiguousarray(A).view(np.float64), device)
+    dB = _dev(np.ascontiguousarray(B).view(np.float64), device)
+    return dA, dB

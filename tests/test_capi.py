@@ -1,0 +1,48 @@
+"""CPU checks of the C ABI: libgtr.so loads and exports every symbol
+include/gtr.h declares; host-only calls work without a GPU."""
+import ctypes
+import os
+import re
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+def declared_symbols():
+    src = open(os.path.join(ROOT, "include", "gtr.h")).read()
+    src = re.sub(r"/\*.*?\*/", "", src, flags=re.S)
+    return sorted(set(re.findall(r"\b(gtr_[a-z0-9_]+)\s*\(", src)))
+
+
+def test_library_exports_every_declared_symbol():
+    from paper_conf_cgo_hubercgtddcd22_b200 import gtr
+    lib = ctypes.CDLL(gtr.LIB_PATH)
+    syms = declared_symbols()
+    assert len(syms) >= 15
+    for s in syms:
+        assert hasattr(lib, s), s
+    assert set(syms) == set(gtr.EXPORTED)
+
+
+def test_host_only_calls():
+    from paper_conf_cgo_hubercgtddcd22_b200 import gtr
+    assert gtr.gtr_version() == 1000
+    assert "heap" in gtr.gtr_strerror(gtr.GTR_EHEAP)
+    assert gtr.gtr_xs_build_workspace_bytes(355, 11303) == 355 * 11303 * 8
+
+
+def test_library_is_sm100a():
+    import subprocess
+    from paper_conf_cgo_hubercgtddcd22_b200 import gtr
+    r = subprocess.run(["cuobjdump", "--list-elf", gtr.LIB_PATH], capture_output=True, text=True)
+    assert r.returncode == 0
+    assert "sm_100a" in r.stdout
+
+
+def test_oracle_is_not_reachable_from_product():
+    pkg = os.path.join(ROOT, "paper_conf_cgo_hubercgtddcd22_b200")
+    for dp, _, fs in os.walk(pkg):
+        for f in fs:
+            if f.endswith((".py", ".cu", ".cuh", ".h")):
+                txt = open(os.path.join(dp, f)).read()
+                assert "import oracle" not in txt and "from oracle" not in txt, f
+                assert "oracle.h" not in txt and "liboracle" not in txt, f

@@ -1,0 +1,59 @@
+"""GPU parity: RS multipole lookup (config 4) vs the oracle.  sin/cos/atan
+differ between glibc and CUDA's libm by about an ulp, so macroscopic XS are
+compared within 1e-12 relative; tallies/hash are exact, guarded by the
+oracle's tie-margin audit."""
+import itertools
+
+import numpy as np
+import pytest
+import torch
+
+import gtr_inputs.rs as RS
+import gtr_inputs.xs as X
+from gpu_common import G, ctx, pool, RUNTIME_MODES, PLACEMENTS  # noqa: F401
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module")
+def rs(orc):
+    t = RS.make_tables()
+    P = orc.RsProblem(t)
+    n = 4000
+    out, v, margin = P.run(1000, n, X.SEED_L, 8, verify=True)
+    assert margin > 1e-10, margin        # no argmax can flip under 1e-12 noise
+    return t, P, out, v, n
+
+
+@pytest.fixture(scope="module")
+def dev(rs):
+    from paper_conf_cgo_hubercgtddcd22_b200.problems import RsDevice
+    return RsDevice(rs[0])
+
+
+def _check(G, ctx, dev, rs, cfg):
+    t, P, o_out, o_v, n = rs
+    out = torch.zeros(18, dtype=torch.uint64, device="cuda")
+    v, bufs = dev.verify_buffers(n)
+    G.gtr_rs_lookup(ctx, cfg, dev.tables, 1000, n, X.SEED_L, out, v)
+    G.gtr_ctx_check(ctx)
+    assert np.array_equal(out.cpu().numpy(), o_out)
+    assert np.array_equal(bufs["mat"].cpu().numpy(), o_v["mat"])
+    assert np.array_equal(bufs["am"].cpu().numpy(), o_v["am"])
+    # 1e-12 relative to the lookup's largest channel: sigE = sigT - sigA can
+    # cancel, so its error is bounded relative to the operands, not the result
+    got, want = bufs["macro"].cpu().numpy(), o_v["macro"]
+    scale = np.abs(want).max(axis=1, keepdims=True)
+    assert (np.abs(got - want) <= 1e-12 * scale).all(), np.abs(got - want).max()
+
+
+@pytest.mark.parametrize("variant", list(itertools.product(RUNTIME_MODES, PLACEMENTS, (0, 1), (128,))),
+                         ids=lambda v: "m%d-p%d-f%d-t%d" % v)
+def test_rs_all_variants(G, ctx, dev, rs, variant):
+    m, p, f, nt = variant
+    _check(G, ctx, dev, rs, G.cfg(m, p, f, nt))
+
+
+@pytest.mark.parametrize("nt", (128, 256))
+def test_rs_native(G, ctx, dev, rs, nt):
+    _check(G, ctx, dev, rs, G.cfg(G.NATIVE, G.PL_STACK, 1, nt))

@@ -1,0 +1,93 @@
+"""GPU parity of the team runtime itself: fork/join (config 2) and the paper's
+semantic programs (Figs. 1, 3, 5, 7, nested parallelism) in every mode,
+placement and fold, against the oracle (exact integers)."""
+import itertools
+
+import numpy as np
+import pytest
+import torch
+
+from gpu_common import G, ctx, pool, RUNTIME_MODES, PLACEMENTS  # noqa: F401
+
+pytestmark = pytest.mark.gpu
+
+FJ_VARIANTS = list(itertools.product(RUNTIME_MODES, PLACEMENTS, (0, 1), (32, 128, 256, 512)))
+
+
+@pytest.mark.parametrize("variant", FJ_VARIANTS, ids=lambda v: "m%d-p%d-f%d-t%d" % v)
+def test_forkjoin_all_variants(G, ctx, orc, variant):
+    m, p, f, nt = variant
+    teams, R = 37, 200
+    for body, K in ((0, 1), (1, 1), (1, 16), (2, 1), (2, 5)):
+        out = torch.zeros(teams, dtype=torch.uint64, device="cuda")
+        G.gtr_forkjoin(ctx, G.cfg(m, p, f, nt, num_teams=teams), R, body, K, out)
+        G.gtr_ctx_check(ctx)
+        got = out.cpu().numpy()
+        want = np.array([orc.fj_team(g, nt, R, body, K) for g in range(teams)], dtype=np.uint64)
+        assert np.array_equal(got, want), (body, K)
+
+
+@pytest.mark.parametrize("pl", PLACEMENTS)
+@pytest.mark.parametrize("nt", (32, 256))
+def test_forkjoin_one_barrier_broadcast(G, ctx, orc, pl, nt):
+    teams, R = 20, 301
+    out = torch.zeros(teams, dtype=torch.uint64, device="cuda")
+    G.gtr_forkjoin(ctx, G.cfg(G.SPMD, pl, 1, nt, num_teams=teams, flags=G.F_BCAST_1BAR), R, 2, 3, out)
+    G.gtr_ctx_check(ctx)
+    want = np.array([orc.fj_team(g, nt, R, 2, 3) for g in range(teams)], dtype=np.uint64)
+    assert np.array_equal(out.cpu().numpy(), want)
+
+
+def test_barrier_floor_runs(G, ctx):
+    out = torch.zeros(148, dtype=torch.uint64, device="cuda")
+    G.gtr_barrier_floor(ctx, G.cfg(thread_limit=256, num_teams=148), 100, out)
+    G.gtr_ctx_check(ctx)
+    assert (out.cpu().numpy() > 0).all()
+
+
+def test_generic_registers_exceed_csm_and_spmd(G):
+    """P:593-597 (fn. 4): function pointers add spurious call edges that raise
+    the register count; the custom state machine removes them."""
+    r = {m: G.gtr_query_variant(G.K_FORKJOIN, G.cfg(m, G.PL_SHARED_STATIC, 1, 128))["regs"]
+         for m in (G.GENERIC, G.GENERIC_CASCADE, G.CSM, G.SPMD)}
+    assert r[G.GENERIC] > r[G.CSM] and r[G.GENERIC_CASCADE] > r[G.CSM], r
+    assert r[G.SPMD] < r[G.GENERIC], r
+
+
+SEM_VARIANTS = list(itertools.product(RUNTIME_MODES, PLACEMENTS, (0, 1), (64, 128)))
+
+
+@pytest.mark.parametrize("variant", SEM_VARIANTS, ids=lambda v: "m%d-p%d-f%d-t%d" % v)
+def test_semantics_all_variants(G, ctx, orc, variant):
+    m, p, f, nt = variant
+    G_teams = 6
+    for test in range(6):
+        if test == 5 and f == 1:
+            continue                       # folding assumes no nested parallelism
+        want = orc.sem_expected(test, G_teams, nt)
+        extra = len(want) if test in (2, 3) else 0
+        out = torch.zeros(len(want) + extra, dtype=torch.uint64, device="cuda")
+        G.gtr_semantics(ctx, G.cfg(m, p, f, nt, num_teams=G_teams), test, out, out.numel())
+        G.gtr_ctx_check(ctx)
+        got = out.cpu().numpy()
+        if test == 1 and p == G.PL_STACK:
+            # Fig. 3 with the locals left in thread-private stack memory: every
+            # thread dereferences thread 0's address in its OWN local window --
+            # the LLVM 12 SPMD miscompile the paper removes.
+            assert np.array_equal(got, want + np.tile(np.arange(nt, dtype=np.uint64), G_teams))
+            continue
+        assert np.array_equal(got[:len(want)], want), test
+        if test in (2, 3):
+            flags = got[len(want):]
+            in_shared = p in (G.PL_RUNTIME, G.PL_SHARED_STATIC, G.PL_STACK)
+            assert (flags == (1 if in_shared else 0)).all(), (test, flags[:4])
+
+
+@pytest.mark.parametrize("pl", PLACEMENTS)
+def test_fig7_separate_guards_same_result(G, ctx, orc, pl):
+    want = orc.sem_expected(4, 6, 64)
+    for flags in (0, G.F_SEPARATE_GUARDS):
+        out = torch.zeros(len(want), dtype=torch.uint64, device="cuda")
+        G.gtr_semantics(ctx, G.cfg(G.SPMD, pl, 1, 64, num_teams=6, flags=flags), 4, out, out.numel())
+        G.gtr_ctx_check(ctx)
+        assert np.array_equal(out.cpu().numpy(), want)

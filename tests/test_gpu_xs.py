@@ -1,0 +1,166 @@
+"""GPU parity: XS lookup (configs 1 and 5) through libgtr.so vs the oracle.
+
+Bar (BASELINE.json north_star): hash, tallies and every integer index
+bit-exact; fp64 macroscopic cross sections within 1e-12 relative -- here they
+are bit-identical, because both sides round every operation separately
+(AMB-12), and the test asserts that.  Results identical across all modes,
+placements and folds.
+"""
+import numpy as np
+import pytest
+import torch
+
+import gtr_inputs.xs as X
+from gpu_common import G, ctx, pool, all_variants, vid  # noqa: F401
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module")
+def small(orc):
+    t = X.make_tables(68)
+    P = orc.XsProblem(t)
+    n = 100000
+    out, v = P.run(0, n, X.SEED_L, 4, verify=True)
+    return t, P, out, v, n
+
+
+@pytest.fixture(scope="module")
+def dev_small(G, ctx, small):
+    from paper_conf_cgo_hubercgtddcd22_b200.problems import XsDevice
+    return XsDevice(ctx, small[0])
+
+
+def test_unionized_grid_matches_oracle(dev_small, small):
+    t, P, *_ = small
+    assert np.array_equal(dev_small.egrid.cpu().numpy(), P.egrid)
+    assert np.array_equal(dev_small.index_grid.cpu().numpy(), P.index_grid)
+
+
+def _run(G, ctx, dev, cfg, first, n, verify=True):
+    out = torch.zeros(18, dtype=torch.uint64, device="cuda")
+    v, bufs = dev.verify_buffers(n) if verify else (None, None)
+    G.gtr_xs_lookup(ctx, cfg, dev.tables, first, n, X.SEED_L, out, v)
+    G.gtr_ctx_check(ctx)
+    return out.cpu().numpy(), ({k: b.cpu().numpy() for k, b in bufs.items()} if verify else None)
+
+
+def _assert_same(out, v, o_out, o_v, lo=0, hi=None):
+    assert np.array_equal(out, o_out)
+    hi = len(o_v["mat"]) if hi is None else hi
+    assert np.array_equal(v["mat"], o_v["mat"][lo:hi])
+    assert np.array_equal(v["u"].astype(np.uint32), o_v["u"][lo:hi])
+    assert np.array_equal(v["am"], o_v["am"][lo:hi])
+    # bit-identical fp64 (stronger than the 1e-12 bar)
+    assert np.array_equal(v["macro"].view(np.uint64), o_v["macro"][lo:hi].view(np.uint64))
+
+
+@pytest.mark.parametrize("variant", all_variants((128, 256)), ids=vid)
+def test_all_variants_bit_exact(G, ctx, dev_small, small, variant):
+    t, P, o_out, o_v, n = small
+    m, p, f, nt = variant
+    out, v = _run(G, ctx, dev_small, G.cfg(m, p, f, nt), 0, n)
+    _assert_same(out, v, o_out, o_v)
+
+
+@pytest.mark.parametrize("nt", (128, 256, 512))
+def test_native_bit_exact(G, ctx, dev_small, small, nt):
+    t, P, o_out, o_v, n = small
+    out, v = _run(G, ctx, dev_small, G.cfg(G.NATIVE, G.PL_STACK, 1, nt), 0, n)
+    _assert_same(out, v, o_out, o_v)
+
+
+@pytest.mark.parametrize("mode", (0, 2, 3, 4))
+@pytest.mark.parametrize("first,n,teams", [(0, 1, 0), (777, 12345, 0), (99991, 9, 3), (5, 70001, 1)])
+def test_ragged_ranges(G, ctx, dev_small, small, orc, mode, first, n, teams):
+    t, P, *_ = small
+    o_out, o_v = P.run(first, n, X.SEED_L, 4, verify=True)
+    out, v = _run(G, ctx, dev_small, G.cfg(mode, G.PL_STACK, 1, 128, num_teams=teams), first, n)
+    _assert_same(out, v, o_out, o_v)
+
+
+def test_empty_request_is_noop(G, ctx, dev_small):
+    out = torch.zeros(18, dtype=torch.uint64, device="cuda")
+    G.gtr_xs_lookup(ctx, G.cfg(), dev_small.tables, 0, 0, X.SEED_L, out)
+    G.gtr_ctx_check(ctx)
+    assert out.cpu().numpy().sum() == 0
+
+
+def test_host_io_entry_point(G, ctx, dev_small, small):
+    t, P, o_out, o_v, n = small
+    h_out = torch.zeros(18, dtype=torch.uint64).pin_memory()
+    req = G.gtr_xs_request(0, n, X.SEED_L)
+    for mode in (G.SPMD, G.NATIVE, G.GENERIC):
+        G.gtr_xs_lookup_host(ctx, G.cfg(mode, G.PL_STACK, 1, 256), dev_small.tables, req, h_out)
+        assert np.array_equal(h_out.numpy(), o_out)
+
+
+def test_runtime_stack_overflow_falls_back_to_pool(G, ctx, dev_small, small):
+    # 16-byte shared stack: most globalized variables spill to the global pool
+    t, P, o_out, o_v, n = small
+    for mode in (G.GENERIC, G.SPMD):
+        out, v = _run(G, ctx, dev_small, G.cfg(mode, G.PL_RUNTIME, 0, 128, smem_stack_bytes=16), 0, n)
+        _assert_same(out, v, o_out, o_v)
+
+
+def test_heap_exhaustion_reports_eheap(G, dev_small):
+    # no fallback pool at all: GTR_PL_GLOBAL cannot allocate -> GTR_EHEAP
+    c = G.gtr_ctx_create(0, None, 0)
+    try:
+        out = torch.zeros(18, dtype=torch.uint64, device="cuda")
+        G.gtr_xs_lookup(c, G.cfg(G.SPMD, G.PL_GLOBAL, 1, 128), dev_small.tables, 0, 1000, X.SEED_L, out)
+        assert G.gtr_ctx_check(c, raise_on_error=False) == G.GTR_EHEAP
+        assert G.gtr_ctx_check(c, raise_on_error=False) == G.GTR_OK     # cleared
+    finally:
+        G.gtr_ctx_destroy(c)
+
+
+def test_invalid_configs_rejected(G, ctx, dev_small):
+    out = torch.zeros(18, dtype=torch.uint64, device="cuda")
+    for bad in (G.cfg(thread_limit=100), G.cfg(mode=7), G.cfg(placement=9), G.cfg(thread_limit=96)):
+        with pytest.raises(G.GtrError):
+            G.gtr_xs_lookup(ctx, bad, dev_small.tables, 0, 10, X.SEED_L, out)
+
+
+def test_duplicate_energies_detected(G, ctx):
+    from paper_conf_cgo_hubercgtddcd22_b200.problems import XsDevice
+    t = X.make_tables(3, 50)
+    t["grid"][1, 10, 0] = t["grid"][0, 20, 0]
+    t["grid"][1] = t["grid"][1][np.argsort(t["grid"][1, :, 0], kind="stable")]
+    with pytest.raises(G.GtrError):
+        XsDevice(ctx, t)
+
+
+def test_variant_resources(G):
+    info = G.gtr_query_variant(G.K_XS, G.cfg(G.SPMD, G.PL_STACK, 1, 256))
+    assert info["block_threads"] == 256 and info["regs"] > 0 and info["num_teams"] > 0
+    gen = G.gtr_query_variant(G.K_XS, G.cfg(G.GENERIC, G.PL_STACK, 1, 256))
+    assert gen["block_threads"] == 288
+
+
+@pytest.mark.slow
+def test_large_config_bench_launch(G, ctx, orc):
+    """Config 5 at full size (355 x 11,303, 17M lookups) in the launch
+    configuration bench.py times: unionized grid exact, sampled index-grid rows
+    exact, hash + tallies of all 17M lookups exact, 20,000 sampled lookups
+    element-wise exact."""
+    from paper_conf_cgo_hubercgtddcd22_b200.problems import XsDevice
+    t = X.make_tables(355)
+    P = orc.XsProblem(t)
+    dev = XsDevice(ctx, t)
+    assert np.array_equal(dev.egrid.cpu().numpy(), P.egrid)
+    rows = np.random.default_rng(3).integers(0, P.n_union, 4000)
+    rows = np.concatenate([rows, [0, 1, P.n_union - 2, P.n_union - 1]])
+    assert np.array_equal(dev.index_grid[torch.from_numpy(rows).cuda()].cpu().numpy(), P.index_grid[rows])
+    n = 17_000_000
+    import os
+    o_out, _ = P.run(0, n, X.SEED_L, os.cpu_count() or 8)
+    for mode in (G.SPMD, G.NATIVE, G.CSM):
+        out = torch.zeros(18, dtype=torch.uint64, device="cuda")
+        G.gtr_xs_lookup(ctx, G.cfg(mode, G.PL_STACK, 1, 256), dev.tables, 0, n, X.SEED_L, out)
+        G.gtr_ctx_check(ctx)
+        assert np.array_equal(out.cpu().numpy(), o_out), mode
+    first, m = 9_876_543, 20000
+    o2, ov = P.run(first, m, X.SEED_L, 8, verify=True)
+    out, v = _run(G, ctx, dev, G.cfg(G.SPMD, G.PL_STACK, 1, 256), first, m)
+    _assert_same(out, v, o2, ov)
