@@ -309,11 +309,13 @@ def sweeps(G, torch, ctx, xs, first, seed, stream):
     out = torch.zeros(18, dtype=torch.uint64, device="cuda")
     modes = {}
     ref = None
-    for name, c in [("native", G.cfg(G.NATIVE, G.PL_STACK, 1, 256)),
-                    ("spmd", G.cfg(G.SPMD, G.PL_STACK, 1, 256)),
-                    ("csm", G.cfg(G.CSM, G.PL_STACK, 1, 256)),
-                    ("cascade", G.cfg(G.GENERIC_CASCADE, G.PL_STACK, 1, 256)),
-                    ("generic", G.cfg(G.GENERIC, G.PL_STACK, 1, 256))]:
+    variants = []
+    for sched, tag in ((0, ""), (G.F_XS_PLAIN, "_plain")):
+        for name, m in (("spmd", G.SPMD), ("csm", G.CSM), ("cascade", G.GENERIC_CASCADE),
+                        ("generic", G.GENERIC)):
+            variants.append((name + tag, G.cfg(m, G.PL_STACK, 1, 256, flags=sched)))
+    variants.insert(0, ("native_plain", G.cfg(G.NATIVE, G.PL_STACK, 1, 256)))
+    for name, c in variants:
         def f():
             out.zero_()
             G.gtr_xs_lookup(ctx, c, xs.tables, first, n, seed, out, None, stream)

@@ -22,12 +22,13 @@ PKG = os.path.dirname(os.path.abspath(__file__))
 CSRC = os.path.join(PKG, "csrc")
 ROOT = os.path.dirname(PKG)
 OBJ = os.path.join(ROOT, "build", "obj")
-LIB = os.path.join(PKG, "libgtr.so")
+LIB = os.environ.get("GTR_LIB_OUT", os.path.join(PKG, "libgtr.so"))
 
 NVCC = os.environ.get("NVCC", shutil.which("nvcc") or "/usr/local/cuda/bin/nvcc")
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 CFLAGS = ARCH + ["-O3", "-std=c++17", "-lineinfo", "-fmad=false", "-Xcompiler", "-fPIC",
                  "-Xcompiler", "-O2", "-I" + os.path.join(ROOT, "include")]
+CFLAGS += os.environ.get("GTR_NVCC_EXTRA", "").split()   # experiments only
 
 # family -> (thread_limits, SPMD-only flag variants)
 FAMILIES = {
@@ -99,11 +100,12 @@ def build(jobs=None, force=False, verbose=True):
     cmd = [NVCC] + ARCH + ["-shared", "-Xlinker", "-z", "-Xlinker", "defs", "-o", LIB + ".tmp"] + objs
     subprocess.check_call(cmd)
     os.replace(LIB + ".tmp", LIB)
-    # drop stale objects of older flag sets
-    keep = set(os.path.basename(o) for o in objs)
-    for f in os.listdir(OBJ):
-        if f.endswith(".o") and f not in keep:
-            os.remove(os.path.join(OBJ, f))
+    # drop stale objects of older flag sets (default build only)
+    if not os.environ.get("GTR_NVCC_EXTRA"):
+        keep = set(os.path.basename(o) for o in objs)
+        for f in os.listdir(OBJ):
+            if f.endswith(".o") and f not in keep:
+                os.remove(os.path.join(OBJ, f))
     if verbose:
         print(f"built {LIB} from {len(objs)} translation units")
     return LIB

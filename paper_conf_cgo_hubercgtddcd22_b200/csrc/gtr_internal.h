@@ -45,7 +45,7 @@ inline uint32_t odd_words(uint32_t bytes) {
 // Compute geometry + runtime params for variant K of kernel `fn`.
 template <class K>
 int resolve(gtr_ctx *ctx, const gtr_launch_cfg *cfg, const void *fn, uint32_t default_stack_bytes,
-            Launch *L, bool stack_always = false) {
+            Launch *L, bool stack_always = false, uint32_t extra_dyn_bytes = 0) {
     L->block = K::BLOCK;
     uint32_t stack_words = 0, stride = 0;
     if (K::PL == PL_RUNTIME || (stack_always && K::PL != PL_GLOBAL)) {
@@ -55,7 +55,10 @@ int resolve(gtr_ctx *ctx, const gtr_launch_cfg *cfg, const void *fn, uint32_t de
         stride = odd_words(bytes);
     }
     L->dyn_smem = tstate_bytes<K>() + (uint32_t)K::BLOCK * stride * 8u;
-    if (L->dyn_smem > 48u * 1024u) {
+    if (extra_dyn_bytes) L->dyn_smem = ((L->dyn_smem + 15u) & ~15u) + extra_dyn_bytes;
+    // static + dynamic above 48 KB needs the opt-in; set it for every launch
+    // with dynamic shared memory (cheap host call)
+    if (L->dyn_smem > 0) {
         if (cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)L->dyn_smem) !=
             cudaSuccess)
             return GTR_EINVAL;

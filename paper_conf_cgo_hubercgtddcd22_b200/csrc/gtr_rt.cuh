@@ -433,6 +433,23 @@ template <class K, class F> __device__ __forceinline__ void for_static(int64_t l
     for (int64_t i = lo + t; i < hi; i += n) body(i);
 }
 
+// `for schedule(dynamic, 32)`: warps claim 32 consecutive iterations at a
+// time from a team counter ("dynamically chosen schedule"); the
+// counter must be zeroed by the sequential code before the region.
+template <class K, class F>
+__device__ __forceinline__ void for_dynamic_warp(int64_t lo, int64_t hi, unsigned int *counter, F &&body) {
+    const unsigned lane = threadIdx.x & 31u;
+    for (;;) {
+        unsigned base = 0;
+        if (lane == 0) base = atomicAdd(counter, 32u);
+        base = __shfl_sync(0xffffffffu, base, 0);
+        const int64_t i = lo + (int64_t)base + lane;
+        if (lo + (int64_t)base >= hi) break;
+        if (i < hi) body(i);
+        __syncwarp();
+    }
+}
+
 // ---------------------------------------------------------------- reductions
 // Team reduction of small integer tallies: shared-memory atomics per event,
 // one global atomic per counter per team at the end.

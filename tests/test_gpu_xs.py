@@ -55,11 +55,12 @@ def _assert_same(out, v, o_out, o_v, lo=0, hi=None):
     assert np.array_equal(v["macro"].view(np.uint64), o_v["macro"][lo:hi].view(np.uint64))
 
 
+@pytest.mark.parametrize("sched", (0, 4), ids=("bucketed", "plain"))
 @pytest.mark.parametrize("variant", all_variants((128, 256)), ids=vid)
-def test_all_variants_bit_exact(G, ctx, dev_small, small, variant):
+def test_all_variants_bit_exact(G, ctx, dev_small, small, variant, sched):
     t, P, o_out, o_v, n = small
     m, p, f, nt = variant
-    out, v = _run(G, ctx, dev_small, G.cfg(m, p, f, nt), 0, n)
+    out, v = _run(G, ctx, dev_small, G.cfg(m, p, f, nt, flags=sched), 0, n)
     _assert_same(out, v, o_out, o_v)
 
 

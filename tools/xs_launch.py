@@ -1,6 +1,6 @@
-"""Launch the XS-large lookup once per requested variant (for ncu captures).
+"""Launch / time the XS-large lookup per variant (ncu captures and A/B timing).
 
-    python tools/xs_launch.py spmd native csm generic [--n 17000000] [--reps 2]
+    python tools/xs_launch.py spmd native ... [--n 17000000] [--reps 3] [--time]
 """
 import argparse
 import os
@@ -18,8 +18,12 @@ from paper_conf_cgo_hubercgtddcd22_b200.problems import XsDevice  # noqa: E402
 VARIANTS = {
     "native": G.cfg(G.NATIVE, G.PL_STACK, 1, 256),
     "spmd": G.cfg(G.SPMD, G.PL_STACK, 1, 256),
+    "spmd128": G.cfg(G.SPMD, G.PL_STACK, 1, 128),
+    "spmd_shared": G.cfg(G.SPMD, G.PL_SHARED_STATIC, 1, 256),
+    "spmd_plain": G.cfg(G.SPMD, G.PL_STACK, 1, 256, flags=G.F_XS_PLAIN),
     "spmd_runtime": G.cfg(G.SPMD, G.PL_RUNTIME, 0, 256),
     "csm": G.cfg(G.CSM, G.PL_STACK, 1, 256),
+    "csm128": G.cfg(G.CSM, G.PL_STACK, 1, 128),
     "generic": G.cfg(G.GENERIC, G.PL_STACK, 1, 256),
 }
 
@@ -28,13 +32,25 @@ ap.add_argument("variants", nargs="+")
 ap.add_argument("--n", type=int, default=17_000_000)
 ap.add_argument("--reps", type=int, default=1)
 ap.add_argument("--niso", type=int, default=355)
+ap.add_argument("--time", action="store_true")
 a = ap.parse_args()
 ctx = G.gtr_ctx_create(0)
 xs = XsDevice(ctx, X.make_tables(a.niso))
 out = torch.zeros(18, dtype=torch.uint64, device="cuda")
 for v in a.variants:
-    for _ in range(a.reps):
-        out.zero_()
-        G.gtr_xs_lookup(ctx, VARIANTS[v], xs.tables, 0, a.n, X.SEED_L, out)
+    c = VARIANTS[v]
+    out.zero_()
+    G.gtr_xs_lookup(ctx, c, xs.tables, 0, a.n, X.SEED_L, out)
+    if a.time:
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record()
+        for _ in range(a.reps):
+            out.zero_()
+            G.gtr_xs_lookup(ctx, c, xs.tables, 0, a.n, X.SEED_L, out)
+        e1.record()
+        torch.cuda.synchronize()
+        ms = e0.elapsed_time(e1) / a.reps
+        info = G.gtr_query_variant(G.K_XS, c)
+        print(f"{v:16s} {ms:8.3f} ms  {a.n / ms / 1e3:8.1f} M lookups/s  regs {info['regs']} "
+              f"teams/SM {info['teams_per_sm']}  hash {int(out.cpu()[0])}", flush=True)
     G.gtr_ctx_check(ctx)
-    print(v, int(out.cpu()[0]))
