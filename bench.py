@@ -36,7 +36,7 @@ BYTES_PER_NUCLIDE = 100     # 4 B index-grid entry + 2 x 48 B gridpoints (SURVEY
 def parse():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
-    ap.add_argument("--steps", type=int, default=10)
+    ap.add_argument("--steps", type=int, default=20)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="gtr", choices=["gtr", "reference"])
     ap.add_argument("--no-sweep", action="store_true", help="skip the per-mode / fork-join sweeps")
@@ -173,7 +173,9 @@ def run_gtr(a):
     xs = XsDevice(ctx, tables, device=dev)
     torch.cuda.synchronize()
     t_setup = time.perf_counter() - t_setup
-    first, n, seed = rank * LOOKUPS_PER_GPU, LOOKUPS_PER_GPU, X.SEED_L
+    from paper_conf_cgo_hubercgtddcd22_b200.dist import shard_range, combine_results, max_over_ranks
+    first, n = shard_range(rank, ws, LOOKUPS_PER_GPU)
+    seed = X.SEED_L
     head = G.cfg(G.SPMD, G.PL_STACK, 1, 256)
     out = torch.zeros(18, dtype=torch.uint64, device=dev)
     num_nucs = tables["num_nucs"].astype(np.int64)
@@ -182,7 +184,7 @@ def run_gtr(a):
         out.zero_()
         G.gtr_xs_lookup(ctx, head, xs.tables, first, n, seed, out, None, stream)
         if dist is not None:
-            dist.all_reduce(out.view(torch.int64), op=dist.ReduceOp.SUM)
+            combine_results(out)
 
     for _ in range(a.warmup):
         step()
@@ -203,7 +205,7 @@ def run_gtr(a):
             G.gtr_xs_lookup(ctx, head, xs.tables, first, n, seed, out, None, stream)
             kev[s][1].record(stream)
             if dist is not None:
-                dist.all_reduce(out.view(torch.int64), op=dist.ReduceOp.SUM)
+                combine_results(out)
         e1.record(stream)
         torch.cuda.synchronize()
         if dist is not None:
@@ -214,7 +216,7 @@ def run_gtr(a):
     res = out.cpu().numpy().astype(np.uint64)
     t_ms = torch.tensor([ms, k_ms], dtype=torch.float64, device=dev)
     if dist is not None:
-        dist.all_reduce(t_ms, op=dist.ReduceOp.MAX)
+        max_over_ranks(t_ms)
     ms, k_ms = float(t_ms[0]), float(t_ms[1])
     value = ws * n / (ms * 1e-3)
 
@@ -225,10 +227,13 @@ def run_gtr(a):
     alg_bytes = alg_bytes_all / ws
     hbm, peak_kind = peaks()
     achieved = alg_bytes / (k_ms * 1e-3) / 1e9
-    traffic = None
-    prof = os.path.join(ROOT, "profiles", "xs_headline_ncu.json")
-    if os.path.exists(prof):
-        traffic = json.load(open(prof)).get("dram_bytes_per_launch")
+    traffic, traffic_src = None, None
+    import glob
+    profs = sorted(glob.glob(os.path.join(ROOT, "profiles", "r*_xs_headline_ncu.json")))
+    if profs:   # dram read+write bytes of the headline kernel from the latest `ncu --set full` capture
+        ks = [k for k in json.load(open(profs[-1]))["kernels"] if "Cfg<3, 3, 1, 256" in k["kernel"]]
+        if ks:
+            traffic, traffic_src = ks[0]["dram_bytes_per_launch"], os.path.relpath(profs[-1], ROOT)
 
     extra = {}
     if rank == 0 and not a.no_sweep:
@@ -246,7 +251,7 @@ def run_gtr(a):
     e2e_s = (time.perf_counter() - t0) / a.steps
     t_e = torch.tensor([e2e_s], dtype=torch.float64, device=dev)
     if dist is not None:
-        dist.all_reduce(t_e, op=dist.ReduceOp.MAX)
+        max_over_ranks(t_e)
     e2e_s = float(t_e[0])
 
     cpu = None
@@ -271,7 +276,7 @@ def run_gtr(a):
                        "table_setup_s": round(t_setup, 2)},
             "hash": int(res[0]), "hash_mod_999983": int(res[0] % 999983),
             "roofline": {"bound": "hbm", "achieved": achieved, "peak": hbm, "unit": "GB/s",
-                         "frac": achieved / hbm, "traffic": traffic,
+                         "frac": achieved / hbm, "traffic": traffic, "traffic_source": traffic_src,
                          "kernel_ms": k_ms, "alg_bytes_per_launch": alg_bytes,
                          "peak_source": f"{peak_kind} MEASURED_PEAKS.json hbm_gbs" if peak_kind == "measured"
                          else "fallback B200_PROFILING.md 6.65 TB/s"},

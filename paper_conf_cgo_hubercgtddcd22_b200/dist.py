@@ -1,0 +1,44 @@
+"""Multi-GPU plumbing for the sharded lookups.
+
+Lookups are independent and defined by their global id, so the N > 1 path is
+a partition of the id range plus one all-reduce of the 18 u64 results (hash +
+12 material tallies + 5 argmax tallies).  Integer sums: the combined result is
+bit-identical for every world size.  torch.distributed supplies the process
+group (NCCL over NVLink on the GPU box, gloo in the CPU tests).
+"""
+import torch
+
+
+def shard_range(rank, world_size, per_rank):
+    """Weak scaling: rank r owns global lookup ids [r*per_rank, (r+1)*per_rank)."""
+    if not (0 <= rank < world_size):
+        raise ValueError("rank out of range")
+    return rank * per_rank, per_rank
+
+
+def split_range(first, n, rank, world_size):
+    """Strong scaling: split [first, first+n) into world_size contiguous parts."""
+    lo = first + n * rank // world_size
+    hi = first + n * (rank + 1) // world_size
+    return lo, hi - lo
+
+
+def combine_results(out, group=None):
+    """All-reduce (SUM) an 18-entry u64 result tensor in place.  u64 is summed
+    through an int64 view: two's-complement addition wraps identically."""
+    import torch.distributed as dist
+    if out.dtype == torch.uint64:
+        view = out.view(torch.int64)
+    elif out.dtype == torch.int64:
+        view = out
+    else:
+        raise TypeError("results must be u64/i64")
+    dist.all_reduce(view, op=dist.ReduceOp.SUM, group=group)
+    return out
+
+
+def max_over_ranks(values, group=None):
+    """Element-wise max of a small float64 tensor over ranks (timings)."""
+    import torch.distributed as dist
+    dist.all_reduce(values, op=dist.ReduceOp.MAX, group=group)
+    return values

@@ -1,0 +1,76 @@
+"""World-size-2 gloo tests of the N > 1 host path: weak-scaling
+shards of the global lookup range, all-reduce of the 18 u64 results.  The
+per-rank results come from the oracle (CPU); the combined hash must equal the
+oracle's over the union of the ranges, for any world size."""
+import os
+import socket
+
+import numpy as np
+import pytest
+import torch
+import torch.multiprocessing as mp
+
+import gtr_inputs.xs as X
+
+
+def _free_port():
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    p = s.getsockname()[1]
+    s.close()
+    return p
+
+
+def _worker(rank, ws, port, per_rank, q):
+    import torch.distributed as dist
+    import oracle
+    from paper_conf_cgo_hubercgtddcd22_b200.dist import shard_range, combine_results, max_over_ranks
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=ws)
+    t = X.make_tables(12, 200, seed_t=5, seed_c=6)
+    P = oracle.XsProblem(t)
+    first, n = shard_range(rank, ws, per_rank)
+    out_np, _ = P.run(first, n, X.SEED_L, 1)
+    out = torch.from_numpy(out_np.copy())           # u64 [18]
+    combine_results(out)
+    tm = max_over_ranks(torch.tensor([float(rank + 1)], dtype=torch.float64))
+    if rank == 0:
+        q.put((out.numpy().copy(), float(tm[0])))
+    dist.destroy_process_group()
+
+
+@pytest.mark.parametrize("ws", [2, 3])
+def test_sharded_hash_equals_union(orc, ws):
+    per_rank = 1500
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_worker, args=(r, ws, port, per_rank, q)) for r in range(ws)]
+    for p in procs:
+        p.start()
+    got, tmax = q.get(timeout=120)
+    for p in procs:
+        p.join(timeout=120)
+        assert p.exitcode == 0
+    t = X.make_tables(12, 200, seed_t=5, seed_c=6)
+    want, _ = orc.XsProblem(t).run(0, ws * per_rank, X.SEED_L, 1)
+    assert np.array_equal(got, want)
+    assert tmax == float(ws)
+
+
+def test_shard_and_split_ranges():
+    from paper_conf_cgo_hubercgtddcd22_b200.dist import shard_range, split_range
+    assert shard_range(3, 8, 17_000_000) == (51_000_000, 17_000_000)
+    parts = [split_range(10, 1001, r, 4) for r in range(4)]
+    assert parts[0][0] == 10 and sum(n for _, n in parts) == 1001
+    assert all(parts[i][0] + parts[i][1] == parts[i + 1][0] for i in range(3))
+    with pytest.raises(ValueError):
+        shard_range(2, 2, 5)
+
+
+def test_u64_wraparound_through_int64_view():
+    # hashes are u64; the int64 view used for the collective must round-trip
+    a = torch.tensor([2 ** 63 + 5], dtype=torch.uint64)
+    v = a.view(torch.int64)
+    assert v.view(torch.uint64)[0] == a[0]
