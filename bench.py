@@ -362,7 +362,60 @@ def sweeps(G, torch, ctx, xs, first, seed, stream):
             row[name + "_regs"] = G.gtr_query_variant(G.K_FORKJOIN, c)["regs"]
         fj[f"thread_limit_{nt}"] = row
     G.gtr_ctx_check(ctx, stream)
-    return {"modes": modes, "ladder_spmd": ladder, "forkjoin": fj}
+    return {"modes": modes, "ladder_spmd": ladder, "forkjoin": fj,
+            "su3": su3_sweep(G, torch, ctx, stream), "rsbench": rs_sweep(G, torch, ctx, stream)}
+
+
+def su3_sweep(G, torch, ctx, stream):
+    """Config 3: SU(3) mat_nn on a 32^4 lattice, fp64; ms per iteration and
+    algorithmic GB/s (1152 B per site: read A 576 + write C 576, B cached)."""
+    import gtr_inputs.su3 as S
+    from paper_conf_cgo_hubercgtddcd22_b200.problems import su3_device
+    sites = 32 ** 4
+    A, B = S.make_lattice(sites, "constant")
+    dA, dB = su3_device(A, B)
+    dC = torch.empty_like(dA)
+    res = {"workload": "32^4 lattice, 4 links/site, complex fp64, constant inputs (C == 1 exactly)"}
+    for name, c in [("native", G.cfg(G.NATIVE, G.PL_STACK, 1, 256)),
+                    ("spmd", G.cfg(G.SPMD, G.PL_STACK, 1, 64)),
+                    ("csm", G.cfg(G.CSM, G.PL_STACK, 1, 64)),
+                    ("cascade", G.cfg(G.GENERIC_CASCADE, G.PL_STACK, 1, 64)),
+                    ("generic", G.cfg(G.GENERIC, G.PL_STACK, 1, 64)),
+                    ("generic_runtime_globalized", G.cfg(G.GENERIC, G.PL_RUNTIME, 0, 64))]:
+        ms = _time(torch, stream, lambda: G.gtr_su3_mat_nn(ctx, c, dA, dB, dC, sites, 1, stream), 3)
+        ok = bool(torch.all(dC.view(-1, 2)[:, 0] == 1.0).item()) and bool(torch.all(dC.view(-1, 2)[:, 1] == 0.0).item())
+        res[name] = {"ms_per_iter": ms, "gb_s": sites * 1152 / (ms * 1e-3) / 1e9,
+                     "regs": G.gtr_query_variant(G.K_SU3, c)["regs"], "closed_form_ok": ok}
+    G.gtr_ctx_check(ctx, stream)
+    del dA, dC
+    return res
+
+
+def rs_sweep(G, torch, ctx, stream, n=2_000_000):
+    """Config 4: RSBench multipole lookups (355 nuclides), lookups/s per mode
+    on the first n of the 10M lookups."""
+    import gtr_inputs.rs as RS
+    import gtr_inputs.xs as X
+    from paper_conf_cgo_hubercgtddcd22_b200.problems import RsDevice
+    dev = RsDevice(RS.make_tables())
+    out = torch.zeros(18, dtype=torch.uint64, device="cuda")
+    res = {"workload": f"355 nuclides, ~1000 poles / 100 windows each, first {n} of 10M lookups"}
+    ref = None
+    for name, c in [("native", G.cfg(G.NATIVE, G.PL_STACK, 1, 128)),
+                    ("spmd", G.cfg(G.SPMD, G.PL_STACK, 1, 128)),
+                    ("csm", G.cfg(G.CSM, G.PL_STACK, 1, 128)),
+                    ("generic", G.cfg(G.GENERIC, G.PL_STACK, 1, 128)),
+                    ("spmd_runtime_globalized", G.cfg(G.SPMD, G.PL_RUNTIME, 0, 128))]:
+        def f():
+            out.zero_()
+            G.gtr_rs_lookup(ctx, c, dev.tables, 0, n, X.SEED_L, out, None, stream)
+        ms = _time(torch, stream, f, 1)
+        r = out.cpu().numpy()
+        ref = r if ref is None else ref
+        res[name] = {"lookups_per_s": n / (ms * 1e-3), "ms": ms, "regs": G.gtr_query_variant(G.K_RS, c)["regs"],
+                     "same_result": bool(np.array_equal(r, ref))}
+    G.gtr_ctx_check(ctx, stream)
+    return res
 
 
 if __name__ == "__main__":
