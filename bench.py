@@ -315,7 +315,7 @@ def sweeps(G, torch, ctx, xs, first, seed, stream):
     modes = {}
     ref = None
     variants = []
-    for sched, tag in ((0, ""), (G.F_XS_PLAIN, "_plain")):
+    for sched, tag in ((0, ""), (G.F_PLAIN, "_plain")):
         for name, m in (("spmd", G.SPMD), ("csm", G.CSM), ("cascade", G.GENERIC_CASCADE),
                         ("generic", G.GENERIC)):
             variants.append((name + tag, G.cfg(m, G.PL_STACK, 1, 256, flags=sched)))
@@ -401,11 +401,14 @@ def rs_sweep(G, torch, ctx, stream, n=2_000_000):
     out = torch.zeros(18, dtype=torch.uint64, device="cuda")
     res = {"workload": f"355 nuclides, ~1000 poles / 100 windows each, first {n} of 10M lookups"}
     ref = None
-    for name, c in [("native", G.cfg(G.NATIVE, G.PL_STACK, 1, 128)),
+    for name, c in [("native_plain", G.cfg(G.NATIVE, G.PL_STACK, 1, 128)),
                     ("spmd", G.cfg(G.SPMD, G.PL_STACK, 1, 128)),
+                    ("spmd_plain", G.cfg(G.SPMD, G.PL_STACK, 1, 128, flags=G.F_PLAIN)),
                     ("csm", G.cfg(G.CSM, G.PL_STACK, 1, 128)),
                     ("generic", G.cfg(G.GENERIC, G.PL_STACK, 1, 128)),
-                    ("spmd_runtime_globalized", G.cfg(G.SPMD, G.PL_RUNTIME, 0, 128))]:
+                    ("generic_plain", G.cfg(G.GENERIC, G.PL_STACK, 1, 128, flags=G.F_PLAIN)),
+                    ("spmd_runtime_globalized", G.cfg(G.SPMD, G.PL_RUNTIME, 0, 128)),
+                    ("spmd_global_heap", G.cfg(G.SPMD, G.PL_GLOBAL, 0, 128))]:
         def f():
             out.zero_()
             G.gtr_rs_lookup(ctx, c, dev.tables, 0, n, X.SEED_L, out, None, stream)

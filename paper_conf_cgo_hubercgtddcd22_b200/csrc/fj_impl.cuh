@@ -89,6 +89,7 @@ template <class K> __device__ __forceinline__ uint64_t team_program() {
     const int body = g_p.body, KK = g_p.K;
     const uint64_t g = (uint64_t)team_num<K>();
     uint64_t count = 0;
+    int kk = 0;                                   // r mod K, kept as a counter
     for (int64_t r = 0; r < R; r++) {
         uint64_t v = 0;
         if (body == 2)
@@ -105,7 +106,8 @@ template <class K> __device__ __forceinline__ uint64_t team_program() {
             x.r = r;
             x.v = v;
         });
-        fork_k<K, 0>((int)(r % KK), args.get());
+        fork_k<K, 0>(kk, args.get());
+        kk = (kk + 1 == KK) ? 0 : kk + 1;
         count += 1;
     }
     return count;

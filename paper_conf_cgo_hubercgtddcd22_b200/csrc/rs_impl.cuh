@@ -30,6 +30,7 @@ struct Params {
     int64_t n_nuc, max_poles, max_windows;
     int32_t max_num_nucs;
     uint32_t chunk;
+    int32_t plain;            // 1: the paper's schedule (GTR_F_PLAIN)
     uint64_t first, n, seed;
     uint8_t *v_mat;
     uint8_t *v_am;
@@ -220,11 +221,65 @@ template <class K> struct LookupRegion {
     }
 };
 
+// Material-bucketed schedule (as XS): fuel lookups evaluate 321
+// nuclides' windows, the others 4-27, so a warp of mixed lookups idles most
+// lanes.  Region 1 samples each lookup's material, the main thread forms
+// buckets, region 2 scatters, region 3 runs whole lookups bucket by bucket
+// with schedule(dynamic, 32).  Per-lookup arithmetic unchanged.
+constexpr uint32_t kBucketLookupsPerThread = 16;
+template <class K> struct ChunkBuf {
+    static constexpr int CH = kBucketLookupsPerThread * K::NT;
+    uint16_t perm[CH];
+    uint8_t mat[CH];
+    uint32_t cnt[12], cur[12];
+    unsigned int next;
+};
+template <class K> __device__ __forceinline__ ChunkBuf<K> &chunk_buf() {
+    const uint32_t off = tstate_bytes<K>() + (uint32_t)K::BLOCK * g_ts.rp.sm_stride_words * 8u;
+    return *reinterpret_cast<ChunkBuf<K> *>(g_dyn + ((off + 15u) & ~15u));
+}
+template <class K> struct SampleRegion {
+    static constexpr int ID = 2;
+    static __device__ void run(void *a) {
+        const Chunk *c = static_cast<const Chunk *>(a);
+        const uint64_t base = c->base, cnt = c->count;
+        ChunkBuf<K> &b = chunk_buf<K>();
+        for_static<K>(0, (int64_t)cnt, [&](int64_t k) {
+            uint64_t s = smp::lcg_jump(g_p.seed, 2ULL * (base + (uint64_t)k));
+            (void)smp::lcg_uniform(s);                  // the energy draw
+            const int m = smp::sample_material(s);
+            b.mat[k] = (uint8_t)m;
+            atomicAdd(&b.cnt[m], 1u);
+        });
+    }
+};
+template <class K> struct ScatterRegion {
+    static constexpr int ID = 3;
+    static __device__ void run(void *a) {
+        const uint64_t cnt = static_cast<const Chunk *>(a)->count;
+        ChunkBuf<K> &b = chunk_buf<K>();
+        for_static<K>(0, (int64_t)cnt, [&](int64_t k) {
+            const uint32_t pos = atomicAdd(&b.cur[b.mat[k]], 1u);
+            b.perm[pos] = (uint16_t)k;
+        });
+    }
+};
+template <class K> struct BucketRegion {
+    static constexpr int ID = 4;
+    static __device__ void run(void *a) {
+        const Chunk *c = static_cast<const Chunk *>(a);
+        const uint64_t base = c->base, cnt = c->count;
+        ChunkBuf<K> &b = chunk_buf<K>();
+        for_dynamic_warp<K>(0, (int64_t)cnt, &b.next,
+                            [&](int64_t q) { lookup<K>(g_p, base + b.perm[q], g_tally); });
+    }
+};
+
 template <class K> __global__ void __launch_bounds__(K::BLOCK) kernel_rt(Params P, RtParams rp) {
     const Role role = team_init<K>(rp);
     if (role == Role::Exit) return;
     if (role == Role::Worker) {
-        worker_loop<K, LookupRegion<K>>();
+        worker_loop<K, LookupRegion<K>, SampleRegion<K>, ScatterRegion<K>, BucketRegion<K>>();
         return;
     }
     guarded<K>([&] {
@@ -239,7 +294,25 @@ template <class K> __global__ void __launch_bounds__(K::BLOCK) kernel_rt(Params 
             x.base = P.first + c * ch;
             x.count = (c * ch + ch <= n) ? ch : n - c * ch;
         });
-        parallel<K, LookupRegion<K>>(chunk.get());
+        if (P.plain) {
+            parallel<K, LookupRegion<K>>(chunk.get());
+            continue;
+        }
+        ChunkBuf<K> &b = chunk_buf<K>();
+        guarded<K>([&] {
+            for (int m = 0; m < 12; m++) b.cnt[m] = 0;
+            b.next = 0;
+        });
+        parallel<K, SampleRegion<K>>(chunk.get());
+        guarded<K>([&] {
+            uint32_t off = 0;
+            for (int m = 0; m < 12; m++) {
+                b.cur[m] = off;
+                off += b.cnt[m];
+            }
+        });
+        parallel<K, ScatterRegion<K>>(chunk.get());
+        parallel<K, BucketRegion<K>>(chunk.get());
     }
     if constexpr (K::MODE == SPMD) flush(g_tally, g_p.out, threadIdx.x, K::NT);
     else flush(g_tally, g_p.out, 0, 1);
@@ -261,14 +334,15 @@ template <class K> struct OpRt {
     static int run(LaunchArgs &a) {
         const void *fn = reinterpret_cast<const void *>(&kernel_rt<K>);
         Launch L;
-        int st = resolve<K>(a.ctx, a.cfg, fn, kDefaultStackBytes, &L);
+        int st = resolve<K>(a.ctx, a.cfg, fn, kDefaultStackBytes, &L, false,
+                            a.P.plain ? 0u : (uint32_t)sizeof(ChunkBuf<K>) + 16u);
         if (st) return st;
         if (a.info) {
             int per_sm = 0;
             GTR_CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, fn, K::BLOCK, L.dyn_smem));
             return fill_info<K>(fn, L, per_sm, a.info);
         }
-        a.P.chunk = kLookupsPerThreadPerChunk * K::NT;
+        a.P.chunk = (a.P.plain ? kLookupsPerThreadPerChunk : kBucketLookupsPerThread) * K::NT;
         kernel_rt<K><<<L.teams, L.block, L.dyn_smem, a.stream>>>(a.P, L.rp);
         GTR_CUDA_TRY(cudaGetLastError());
         return GTR_OK;

@@ -104,7 +104,7 @@ template <int NT> int run_native(LaunchArgs &a) {
 inline int launch(LaunchArgs &a) {
     const gtr_launch_cfg *c = a.cfg;
     if (!valid_cfg(c)) return GTR_EINVAL;
-    a.P.plain = (c->flags & GTR_F_XS_PLAIN) ? 1 : 0;
+    a.P.plain = (c->flags & GTR_F_PLAIN) ? 1 : 0;
     if (c->mode == NATIVE) {
         if (c->thread_limit == 128) return run_native<128>(a);
         if (c->thread_limit == 256) return run_native<256>(a);

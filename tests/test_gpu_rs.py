@@ -47,11 +47,12 @@ def _check(G, ctx, dev, rs, cfg):
     assert (np.abs(got - want) <= 1e-12 * scale).all(), np.abs(got - want).max()
 
 
+@pytest.mark.parametrize("sched", (0, 4), ids=("bucketed", "plain"))
 @pytest.mark.parametrize("variant", list(itertools.product(RUNTIME_MODES, PLACEMENTS, (0, 1), (128,))),
                          ids=lambda v: "m%d-p%d-f%d-t%d" % v)
-def test_rs_all_variants(G, ctx, dev, rs, variant):
+def test_rs_all_variants(G, ctx, dev, rs, variant, sched):
     m, p, f, nt = variant
-    _check(G, ctx, dev, rs, G.cfg(m, p, f, nt))
+    _check(G, ctx, dev, rs, G.cfg(m, p, f, nt, flags=sched))
 
 
 @pytest.mark.parametrize("nt", (128, 256))

@@ -20,7 +20,7 @@ VARIANTS = {
     "spmd": G.cfg(G.SPMD, G.PL_STACK, 1, 256),
     "spmd128": G.cfg(G.SPMD, G.PL_STACK, 1, 128),
     "spmd_shared": G.cfg(G.SPMD, G.PL_SHARED_STATIC, 1, 256),
-    "spmd_plain": G.cfg(G.SPMD, G.PL_STACK, 1, 256, flags=G.F_XS_PLAIN),
+    "spmd_plain": G.cfg(G.SPMD, G.PL_STACK, 1, 256, flags=G.F_PLAIN),
     "spmd_runtime": G.cfg(G.SPMD, G.PL_RUNTIME, 0, 256),
     "csm": G.cfg(G.CSM, G.PL_STACK, 1, 256),
     "csm128": G.cfg(G.CSM, G.PL_STACK, 1, 128),
