@@ -91,3 +91,27 @@ extern "C" int gtr_query_variant(int kernel, const gtr_launch_cfg *cfg, gtr_vari
     default: return GTR_EINVAL;
     }
 }
+
+extern "C" int gtr_l2_persist(gtr_ctx *c, const void *base, uint64_t bytes, uint64_t persist_bytes, float hit_ratio,
+                              void *stream) {
+    if (!c || hit_ratio < 0.f || hit_ratio > 1.f || (bytes && !base)) return GTR_EINVAL;
+    cudaStream_t s = static_cast<cudaStream_t>(stream);
+    cudaStreamAttrValue v = {};
+    if (bytes) {
+        int max_persist = 0, max_window = 0;
+        GTR_CUDA_TRY(cudaDeviceGetAttribute(&max_persist, cudaDevAttrMaxPersistingL2CacheSize, c->device));
+        GTR_CUDA_TRY(cudaDeviceGetAttribute(&max_window, cudaDevAttrMaxAccessPolicyWindowSize, c->device));
+        uint64_t lim = persist_bytes < (uint64_t)max_persist ? persist_bytes : (uint64_t)max_persist;
+        GTR_CUDA_TRY(cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, lim));
+        v.accessPolicyWindow.base_ptr = const_cast<void *>(base);
+        v.accessPolicyWindow.num_bytes = bytes < (uint64_t)max_window ? bytes : (uint64_t)max_window;
+        v.accessPolicyWindow.hitRatio = hit_ratio;
+        v.accessPolicyWindow.hitProp = cudaAccessPropertyPersisting;
+        v.accessPolicyWindow.missProp = cudaAccessPropertyStreaming;
+    } else {
+        v.accessPolicyWindow.num_bytes = 0;
+        GTR_CUDA_TRY(cudaCtxResetPersistingL2Cache());
+    }
+    GTR_CUDA_TRY(cudaStreamSetAttribute(s, cudaStreamAttributeAccessPolicyWindow, &v));
+    return GTR_OK;
+}

@@ -95,6 +95,7 @@ _proto = {
     "gtr_xs_lookup": (_i, [_vp, _P(gtr_launch_cfg), _P(gtr_xs_tables), _u64, _u64, _u64, _vp,
                            _P(gtr_xs_verify), _vp]),
     "gtr_xs_lookup_host": (_i, [_vp, _P(gtr_launch_cfg), _P(gtr_xs_tables), _P(gtr_xs_request), _vp, _vp]),
+    "gtr_l2_persist": (_i, [_vp, _vp, _u64, _u64, C.c_float, _vp]),
     "gtr_su3_mat_nn": (_i, [_vp, _P(gtr_launch_cfg), _vp, _vp, _vp, _i64, C.c_int32, _vp]),
     "gtr_rs_lookup": (_i, [_vp, _P(gtr_launch_cfg), _P(gtr_rs_tables), _u64, _u64, _u64, _vp,
                            _P(gtr_rs_verify), _vp]),
@@ -209,3 +210,8 @@ def gtr_rs_lookup(ctx, launch_cfg, tables, first, n, seed, d_out, verify=None, s
     return _check("gtr_rs_lookup", _lib.gtr_rs_lookup(ctx, C.byref(launch_cfg), C.byref(tables), first, n, seed,
                                                       _ptr(d_out), C.byref(verify) if verify else None,
                                                       _stream(stream)))
+
+
+def gtr_l2_persist(ctx, d_base, nbytes, persist_bytes, hit_ratio, stream=None):
+    return _check("gtr_l2_persist", _lib.gtr_l2_persist(ctx, _ptr(d_base), nbytes, persist_bytes, hit_ratio,
+                                                        _stream(stream)))

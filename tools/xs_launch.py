@@ -33,10 +33,15 @@ ap.add_argument("--n", type=int, default=17_000_000)
 ap.add_argument("--reps", type=int, default=1)
 ap.add_argument("--niso", type=int, default=355)
 ap.add_argument("--time", action="store_true")
+ap.add_argument("--persist", type=float, default=0.0, help="L2 persisting window over the grid, hit ratio")
+ap.add_argument("--persist-mb", type=int, default=96)
 a = ap.parse_args()
 ctx = G.gtr_ctx_create(0)
 xs = XsDevice(ctx, X.make_tables(a.niso))
 out = torch.zeros(18, dtype=torch.uint64, device="cuda")
+if a.persist > 0:
+    G.gtr_l2_persist(ctx, xs.grid, xs.grid.numel() * 8, a.persist_mb << 20, a.persist)
+    print("persist window", a.persist, a.persist_mb, "MB")
 for v in a.variants:
     c = VARIANTS[v]
     out.zero_()
