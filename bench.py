@@ -333,7 +333,8 @@ def sweeps(G, torch, ctx, xs, first, seed, stream):
                        "teams_per_sm": info["teams_per_sm"], "same_result": bool(np.array_equal(r, ref))}
     # the paper's ladder (Fig. 11a) on SPMD: globalized at runtime -> h2s2 -> +fold
     ladder = {}
-    for name, c in [("runtime_globalized", G.cfg(G.SPMD, G.PL_RUNTIME, 0, 256)),
+    for name, c in [("llvm12_coalesced", G.cfg(G.SPMD, G.PL_COALESCED, 0, 256)),
+                    ("runtime_globalized", G.cfg(G.SPMD, G.PL_RUNTIME, 0, 256)),
                     ("global_heap", G.cfg(G.SPMD, G.PL_GLOBAL, 0, 256)),
                     ("heap_to_shared", G.cfg(G.SPMD, G.PL_SHARED_STATIC, 0, 256)),
                     ("heap_to_stack", G.cfg(G.SPMD, G.PL_STACK, 0, 256)),
@@ -354,12 +355,27 @@ def sweeps(G, torch, ctx, xs, first, seed, stream):
         fl = G.cfg(thread_limit=nt, num_teams=teams)
         row["barrier_floor_ns"] = _time(torch, stream, lambda: G.gtr_barrier_floor(ctx, fl, R, fo, stream), 2) \
             * 1e6 / R
-        for name, m, flags in [("generic", G.GENERIC, 0), ("cascade", G.GENERIC_CASCADE, 0),
-                               ("csm", G.CSM, 0), ("spmd", G.SPMD, 0)]:
-            c = G.cfg(m, G.PL_SHARED_STATIC, 1, nt, num_teams=teams, flags=flags)
+        # trivial body, K = 4 distinct regions, region args in static shared
+        # memory (heap-to-shared) for every mode; spmd_stack privatizes them
+        # (heap-to-stack: no guard barrier)
+        for name, m, pl in [("generic", G.GENERIC, G.PL_SHARED_STATIC),
+                            ("cascade", G.GENERIC_CASCADE, G.PL_SHARED_STATIC),
+                            ("csm", G.CSM, G.PL_SHARED_STATIC), ("spmd", G.SPMD, G.PL_SHARED_STATIC),
+                            ("spmd_stack", G.SPMD, G.PL_STACK),
+                            ("generic_runtime_nofold", G.GENERIC, G.PL_RUNTIME)]:
+            c = G.cfg(m, pl, 0 if name.endswith("nofold") else 1, nt, num_teams=teams)
             ms = _time(torch, stream, lambda: G.gtr_forkjoin(ctx, c, R, 1, 4, fo, stream), 2)
             row[name + "_ns"] = ms * 1e6 / R
             row[name + "_regs"] = G.gtr_query_variant(G.K_FORKJOIN, c)["regs"]
+        # broadcast body (a guarded side effect producing a value): 2-barrier
+        # broadcast vs the double-buffered 1-barrier form
+        for name, flags in [("spmd_bcast_2bar", 0), ("spmd_bcast_1bar", G.F_BCAST_1BAR)]:
+            c = G.cfg(G.SPMD, G.PL_STACK, 1, nt, num_teams=teams, flags=flags)
+            ms = _time(torch, stream, lambda: G.gtr_forkjoin(ctx, c, R, 2, 1, fo, stream), 2)
+            row[name + "_ns"] = ms * 1e6 / R
+        c = G.cfg(G.GENERIC, G.PL_STACK, 1, nt, num_teams=teams)
+        row["generic_bcast_ns"] = _time(torch, stream, lambda: G.gtr_forkjoin(ctx, c, R, 2, 1, fo, stream), 2) \
+            * 1e6 / R
         fj[f"thread_limit_{nt}"] = row
     G.gtr_ctx_check(ctx, stream)
     return {"modes": modes, "ladder_spmd": ladder, "forkjoin": fj,
@@ -381,7 +397,9 @@ def su3_sweep(G, torch, ctx, stream):
                     ("csm", G.cfg(G.CSM, G.PL_STACK, 1, 64)),
                     ("cascade", G.cfg(G.GENERIC_CASCADE, G.PL_STACK, 1, 64)),
                     ("generic", G.cfg(G.GENERIC, G.PL_STACK, 1, 64)),
-                    ("generic_runtime_globalized", G.cfg(G.GENERIC, G.PL_RUNTIME, 0, 64))]:
+                    ("generic_runtime_globalized", G.cfg(G.GENERIC, G.PL_RUNTIME, 0, 64)),
+                    ("generic_llvm12_coalesced", G.cfg(G.GENERIC, G.PL_COALESCED, 0, 64)),
+                    ("csm_shared_fold", G.cfg(G.CSM, G.PL_SHARED_STATIC, 1, 64))]:
         ms = _time(torch, stream, lambda: G.gtr_su3_mat_nn(ctx, c, dA, dB, dC, sites, 1, stream), 3)
         ok = bool(torch.all(dC.view(-1, 2)[:, 0] == 1.0).item()) and bool(torch.all(dC.view(-1, 2)[:, 1] == 0.0).item())
         res[name] = {"ms_per_iter": ms, "gb_s": sites * 1152 / (ms * 1e-3) / 1e9,

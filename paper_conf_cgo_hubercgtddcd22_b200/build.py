@@ -48,7 +48,7 @@ def units():
         src = fam + "_variant.cu"
         for nt in nts:
             for mode in (0, 1):
-                for pl in range(4):
+                for pl in range(5):
                     for fold in (0, 1):
                         out.append((f"{fam}_m{mode}_p{pl}_f{fold}_t{nt}", src,
                                     [f"-DGTR_V_MODE={mode}", f"-DGTR_V_PL={pl}",

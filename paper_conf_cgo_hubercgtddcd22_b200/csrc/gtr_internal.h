@@ -48,7 +48,7 @@ int resolve(gtr_ctx *ctx, const gtr_launch_cfg *cfg, const void *fn, uint32_t de
             Launch *L, bool stack_always = false, uint32_t extra_dyn_bytes = 0) {
     L->block = K::BLOCK;
     uint32_t stack_words = 0, stride = 0;
-    if (K::PL == PL_RUNTIME || (stack_always && K::PL != PL_GLOBAL)) {
+    if (K::PL == PL_RUNTIME || K::PL == PL_COALESCED || (stack_always && K::PL != PL_GLOBAL)) {
         uint32_t bytes = cfg->smem_stack_bytes ? cfg->smem_stack_bytes : default_stack_bytes;
         stack_words = (bytes + 7u) / 8u;
         if (stack_words > 4095u) return GTR_EINVAL;
@@ -99,7 +99,8 @@ int dispatch_mpf(int mode, int pl, int fold, A &&...a) {
         return Op<Cfg<M, P, false, NT, FLAGS>>::run(a...);                                 \
     }
 #define GTR_CASES(M)                                                                       \
-    GTR_CASE(M, PL_RUNTIME) GTR_CASE(M, PL_GLOBAL) GTR_CASE(M, PL_SHARED_STATIC) GTR_CASE(M, PL_STACK)
+    GTR_CASE(M, PL_RUNTIME) GTR_CASE(M, PL_GLOBAL) GTR_CASE(M, PL_SHARED_STATIC) GTR_CASE(M, PL_STACK) \
+    GTR_CASE(M, PL_COALESCED)
     GTR_CASES(GENERIC)
     GTR_CASES(GENERIC_CASCADE)
     GTR_CASES(CSM)
@@ -117,7 +118,7 @@ int dispatch_spmd(int pl, int fold, A &&...a) {
         if (fold) return Op<Cfg<SPMD, P, true, NT, FLAGS>>::run(a...);                     \
         return Op<Cfg<SPMD, P, false, NT, FLAGS>>::run(a...);                              \
     }
-    GTR_CASE(PL_RUNTIME) GTR_CASE(PL_GLOBAL) GTR_CASE(PL_SHARED_STATIC) GTR_CASE(PL_STACK)
+    GTR_CASE(PL_RUNTIME) GTR_CASE(PL_GLOBAL) GTR_CASE(PL_SHARED_STATIC) GTR_CASE(PL_STACK) GTR_CASE(PL_COALESCED)
 #undef GTR_CASE
     return GTR_EUNSUPPORTED;
 }
@@ -125,7 +126,7 @@ int dispatch_spmd(int pl, int fold, A &&...a) {
 inline bool valid_cfg(const gtr_launch_cfg *c) {
     if (!c) return false;
     if (c->mode < 0 || c->mode > 4) return false;
-    if (c->placement < 0 || c->placement > 3) return false;
+    if (c->placement < 0 || c->placement > 4) return false;
     if (c->thread_limit <= 0 || c->thread_limit % 32 != 0) return false;
     if (c->num_teams < 0) return false;
     return true;

@@ -27,6 +27,11 @@
 //   PL_SHARED_STATIC  heap-to-shared: static __shared__ storage;
 //                     per-thread variables scaled by the thread count (Fig. 6b)
 //   PL_STACK          heap-to-stack: registers / local memory
+//   PL_COALESCED      LLVM 12's globalization (Fig. 4b): one
+//                     __runtime_coalesced_alloc per warp, every lane's copy at
+//                     lane stride inside active parallel regions, runtime
+//                     is_spmd / in_active_parallel checks, and the unsound
+//                     SPMD shortcut to thread-private memory
 //
 // Runtime-call folding: with FOLD the execution-mode, parallel-
 // level, thread-count and launch-parameter queries are compile-time constants;
@@ -38,7 +43,7 @@
 namespace gtr {
 
 enum : int { GENERIC = 0, GENERIC_CASCADE = 1, CSM = 2, SPMD = 3, NATIVE = 4 };
-enum : int { PL_RUNTIME = 0, PL_GLOBAL = 1, PL_SHARED_STATIC = 2, PL_STACK = 3 };
+enum : int { PL_RUNTIME = 0, PL_GLOBAL = 1, PL_SHARED_STATIC = 2, PL_STACK = 3, PL_COALESCED = 4 };
 enum : uint32_t { ERR_HEAP = 1u, ERR_LIFO = 2u, ERR_DUP_ENERGY = 4u, ERR_BUILD = 8u };
 enum : int { F_BCAST_1BAR = 1, F_SEPARATE_GUARDS = 2 };
 
@@ -88,6 +93,13 @@ struct ThreadState {
     uint8_t nested;   // serialized nested parallel depth
     uint8_t level;    // SPMD: this thread's parallel level
     uint32_t gsp;     // global fallback stack top (words)
+    // PL_COALESCED (per warp, kept in the warp's lane states)
+    uint32_t igsp;    // this lane's own global stack top (divergent calls)
+    uint32_t frame;   // frame slot k lives in lane k: live lanes << 16 | global << 15 | words
+    uint32_t wtop;    // lane 0: warp stack top in shared memory (words)
+    uint32_t wgtop;   // lane 0: warp slab top in the fallback pool (words)
+    uint32_t nframes; // lane 0: frames on the warp stack
+    uint32_t pad;
 };
 extern __shared__ __align__(16) uint8_t g_dyn[];
 
@@ -167,7 +179,7 @@ enum class Role { Main, Worker, Exit };
 // code, guarded).
 template <class K> __device__ __forceinline__ Role team_init(const RtParams &rp) {
     if constexpr (K::TSTATE) {
-        ThreadState z = {0, 0, 0, 0};
+        ThreadState z = {0, 0, 0, 0, 0, 0, 0, 0, 0, 0};
         tstate<K>() = z;
     }
     if constexpr (K::GENERIC_LIKE) {
@@ -338,6 +350,95 @@ template <class K> __device__ __noinline__ void free_shared(void *p, uint32_t by
     }
 }
 
+// __runtime_coalesced_alloc / _free (LLVM 12, Fig. 4b).  A converged warp
+// (all 32 lanes in `mask`) allocates once on a warp stack: its 32 per-thread
+// stack slices (overflow: the warp's slab of the first half of the fallback
+// pool).  Each allocation is a frame with a count of live lanes; a lane's free
+// decrements it, and the lane that releases a frame last pops every fully
+// released frame from the top -- lanes that diverge after the allocation can
+// release it at different times.  Calls from a partial warp (divergent lanes)
+// allocate a per-lane copy from the second half of the pool (LIFO per lane).
+// `words` is the whole allocation (already x32 for a converged parallel warp);
+// `fk` returns the frame index (-1 for a per-lane copy).
+template <class K> __device__ __forceinline__ ThreadState *warp_states() {
+    return reinterpret_cast<ThreadState *>(g_dyn) + (threadIdx.x & ~31u);
+}
+template <class K> __device__ __noinline__ void *alloc_coalesced(uint32_t words, unsigned mask, int &fk) {
+    const RtParams &rp = g_ts.rp;
+    const uint64_t half = rp.pool_wpt / 2;
+    if (mask != 0xffffffffu) {                            // divergent: per-lane copy
+        ThreadState &ts = tstate<K>();
+        fk = -1;
+        if (rp.pool != nullptr && (uint64_t)ts.igsp + words <= half) {
+            uint64_t *p = rp.pool + (uint64_t)gridDim.x * K::BLOCK * half +
+                          ((uint64_t)blockIdx.x * K::BLOCK + threadIdx.x) * half + ts.igsp;
+            ts.igsp += words;
+            return p;
+        }
+        atomicOr(rp.err, (uint32_t)ERR_HEAP);
+        return &g_sink_dummy;
+    }
+    uint64_t *p = nullptr;
+    int k = -1;
+    if ((threadIdx.x & 31u) == 0) {
+        ThreadState *W = warp_states<K>();
+        const uint32_t cap = min(32u * rp.sm_stride_words, 32767u);
+        const uint32_t wbase = threadIdx.x & ~31u;
+        k = (int)W[0].nframes;
+        uint32_t glob = 0;
+        if (k >= 32 || words > 32767u) {
+            k = -1;
+        } else if (W[0].wtop + words <= cap) {
+            p = sm_stack_base<K>() + (size_t)wbase * rp.sm_stride_words + W[0].wtop;
+            W[0].wtop += words;
+        } else if (rp.pool != nullptr && (uint64_t)W[0].wgtop + words <= 32u * half) {
+            p = rp.pool + ((uint64_t)blockIdx.x * K::BLOCK + wbase) * half + W[0].wgtop;
+            W[0].wgtop += words;
+            glob = 0x8000u;
+        } else {
+            k = -1;
+        }
+        if (k < 0) {
+            atomicOr(rp.err, (uint32_t)ERR_HEAP);
+            p = &g_sink_dummy;
+        } else {
+            W[k].frame = (32u << 16) | glob | words;
+            __threadfence_block();
+            W[0].nframes = (uint32_t)k + 1u;
+        }
+    }
+    fk = __shfl_sync(0xffffffffu, k, 0);
+    return reinterpret_cast<void *>(__shfl_sync(0xffffffffu, reinterpret_cast<uintptr_t>(p), 0));
+}
+template <class K> __device__ __noinline__ void free_coalesced(void *p, uint32_t words, int fk) {
+    if (p == &g_sink_dummy) return;
+    if (fk < 0) {
+        tstate<K>().igsp -= words;
+        return;
+    }
+    ThreadState *W = warp_states<K>();
+    __threadfence_block();                                // this lane's uses happen before release
+    const uint32_t old = atomicSub(&W[fk].frame, 1u << 16);
+    if ((old >> 16) != 1u) return;                        // other lanes still use frame fk
+    for (;;) {                                            // pop fully released frames
+        const uint32_t n = *reinterpret_cast<volatile uint32_t *>(&W[0].nframes);
+        if (n == 0) break;
+        const uint32_t f = *reinterpret_cast<volatile uint32_t *>(&W[n - 1].frame);
+        if ((f >> 16) != 0u) break;
+        if (atomicCAS(&W[0].nframes, n, n - 1) != n) continue;
+        if (f & 0x8000u) atomicSub(&W[0].wgtop, f & 0x7fffu);
+        else atomicSub(&W[0].wtop, f & 0x7fffu);
+    }
+    __threadfence_block();
+}
+// the runtime (never folded) queries LLVM 12's lowering evaluates
+template <class K> __device__ __forceinline__ bool rt_is_spmd() { return g_ts.exec_mode == SPMD; }
+template <class K> __device__ __forceinline__ bool rt_in_active_parallel() {
+    const int lvl = (K::MODE == SPMD) ? tstate<K>().level
+                                      : ((int)threadIdx.x == K::MAIN_HW ? 0 : g_ts.level);
+    return lvl == 1 && tstate<K>().nested == 0;
+}
+
 template <int N_WORDS> struct OddStride {
     static constexpr int value = (N_WORDS % 2 == 1) ? N_WORDS : N_WORDS + 1;
 };
@@ -360,6 +461,30 @@ template <class K, class T, int N, class Tag> struct Local<K, T, N, Tag, PL_RUNT
 };
 template <class K, class T, int N, class Tag> struct Local<K, T, N, Tag, PL_GLOBAL>
     : Local<K, T, N, Tag, PL_RUNTIME> {};
+template <class K, class T, int N, class Tag> struct Local<K, T, N, Tag, PL_COALESCED> {
+    static constexpr uint32_t WORDS = (uint32_t)((N * sizeof(T) + 7) / 8);
+    T v[N];
+    T *p;
+    uint32_t words;
+    int fk;
+    __device__ __forceinline__ Local() {
+        if (rt_is_spmd<K>()) {                            // LLVM 12: no globalization in SPMD
+            p = v;
+            words = 0;
+        } else {
+            const unsigned mask = __activemask();
+            const bool par = rt_in_active_parallel<K>() && mask == 0xffffffffu;   // SoA over the warp
+            words = par ? 32u * WORDS : WORDS;
+            uint64_t *base = static_cast<uint64_t *>(alloc_coalesced<K>(words, mask, fk));
+            p = reinterpret_cast<T *>(par ? base + (threadIdx.x & 31u) * WORDS : base);
+        }
+    }
+    __device__ __forceinline__ ~Local() {
+        if (words) free_coalesced<K>(p, words, fk);
+    }
+    __device__ __forceinline__ T &operator[](int i) { return p[i]; }
+    __device__ __forceinline__ T *ptr() { return p; }
+};
 template <class K, class T, int N, class Tag> struct Local<K, T, N, Tag, PL_SHARED_STATIC> {
     static constexpr int WORDS = (int)((N * sizeof(T) + 7) / 8);
     static constexpr int STRIDE = OddStride<WORDS>::value;
@@ -389,7 +514,24 @@ template <class K, class T, int N, class Tag> struct Local<K, T, N, Tag, PL_SHAR
 // cannot privatize it and uses static shared memory instead.
 template <class K, class T, class Tag, bool RO = true> struct TeamLocal {
     static constexpr bool PRIVATE = (K::MODE == SPMD && K::PL == PL_STACK && RO);
-    static constexpr bool RUNTIME_ALLOC = (K::PL == PL_RUNTIME || K::PL == PL_GLOBAL);
+    static constexpr bool RUNTIME_ALLOC = (K::PL == PL_RUNTIME || K::PL == PL_GLOBAL || K::PL == PL_COALESCED);
+    // one copy, allocated in sequential context (coalesced: a single-lane
+    // warp allocation, as LLVM 12 does outside parallel regions)
+    // (coalesced: sequential context -> a single-lane call -> per-lane copy)
+    __device__ __forceinline__ static T *alloc_one() {
+        if constexpr (K::PL == PL_COALESCED) {
+            int fk;
+            return static_cast<T *>(alloc_coalesced<K>((uint32_t)((sizeof(T) + 7) / 8), 1u, fk));
+        } else {
+            return static_cast<T *>(alloc_shared<K>(sizeof(T)));
+        }
+    }
+    __device__ __forceinline__ static void free_one(T *q) {
+        if constexpr (K::PL == PL_COALESCED)
+            free_coalesced<K>(q, (uint32_t)((sizeof(T) + 7) / 8), -1);
+        else
+            free_shared<K>(q, sizeof(T));
+    }
     T priv;
     T *p;
     __device__ __forceinline__ static T *static_slot() {
@@ -401,9 +543,9 @@ template <class K, class T, class Tag, bool RO = true> struct TeamLocal {
             p = &priv;
         } else if constexpr (RUNTIME_ALLOC) {
             if constexpr (K::MODE == SPMD)
-                p = guarded_bcast<K, T *>([] { return static_cast<T *>(alloc_shared<K>(sizeof(T))); });
+                p = guarded_bcast<K, T *>([] { return alloc_one(); });
             else
-                p = static_cast<T *>(alloc_shared<K>(sizeof(T)));
+                p = alloc_one();
         } else {
             p = static_slot();
         }
@@ -412,9 +554,9 @@ template <class K, class T, class Tag, bool RO = true> struct TeamLocal {
         if constexpr (RUNTIME_ALLOC) {
             if constexpr (K::MODE == SPMD) {
                 __syncthreads();
-                if (threadIdx.x == 0) free_shared<K>(p, sizeof(T));
+                if (threadIdx.x == 0) free_one(p);
             } else {
-                free_shared<K>(p, sizeof(T));
+                free_one(p);
             }
         }
     }

@@ -15,7 +15,8 @@
     GTR_INST(M, P, false, GTR_V_GROUP_NT, GTR_V_FLAGS)
 #define GTR_GROUP_M(M)                                                        \
     GTR_GROUP_PL(M, gtr::PL_RUNTIME) GTR_GROUP_PL(M, gtr::PL_GLOBAL)           \
-    GTR_GROUP_PL(M, gtr::PL_SHARED_STATIC) GTR_GROUP_PL(M, gtr::PL_STACK)
+    GTR_GROUP_PL(M, gtr::PL_SHARED_STATIC) GTR_GROUP_PL(M, gtr::PL_STACK)  \
+    GTR_GROUP_PL(M, gtr::PL_COALESCED)
 #if defined(GTR_V_SPMD_ONLY)
 #define GTR_VARIANT_INSTANCES GTR_GROUP_M(gtr::SPMD)
 #else

@@ -4,7 +4,7 @@ import itertools
 import pytest
 
 RUNTIME_MODES = (0, 1, 2, 3)       # GENERIC, CASCADE, CSM, SPMD
-PLACEMENTS = (0, 1, 2, 3)          # RUNTIME, GLOBAL, SHARED_STATIC, STACK
+PLACEMENTS = (0, 1, 2, 3, 4)       # RUNTIME, GLOBAL, SHARED_STATIC, STACK, COALESCED (LLVM 12)
 
 
 def all_variants(nts):

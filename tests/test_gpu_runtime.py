@@ -70,16 +70,22 @@ def test_semantics_all_variants(G, ctx, orc, variant):
         G.gtr_semantics(ctx, G.cfg(m, p, f, nt, num_teams=G_teams), test, out, out.numel())
         G.gtr_ctx_check(ctx)
         got = out.cpu().numpy()
-        if test == 1 and p == G.PL_STACK:
-            # Fig. 3 with the locals left in thread-private stack memory: every
-            # thread dereferences thread 0's address in its OWN local window --
-            # the LLVM 12 SPMD miscompile the paper removes.
+        private = p == G.PL_STACK or (p == G.PL_COALESCED and m == G.SPMD)
+        if test == 1 and private:
+            # Fig. 3 with the locals left in thread-private stack memory (heap-
+            # to-stack, or LLVM 12's SPMD shortcut): every thread dereferences
+            # thread 0's address in its OWN local window -- the miscompile the
+            # paper removes.
             assert np.array_equal(got, want + np.tile(np.arange(nt, dtype=np.uint64), G_teams))
             continue
         assert np.array_equal(got[:len(want)], want), test
         if test in (2, 3):
             flags = got[len(want):]
-            in_shared = p in (G.PL_RUNTIME, G.PL_SHARED_STATIC, G.PL_STACK)
+            # LLVM 12 scheme: a converged warp in a parallel region (Fig. 5c)
+            # gets a warp SoA on the shared-memory warp stack; the lone main
+            # thread (Fig. 5b) and SPMD (private shortcut) do not
+            in_shared = p in (G.PL_RUNTIME, G.PL_SHARED_STATIC, G.PL_STACK) or (
+                p == G.PL_COALESCED and m != G.SPMD and test == 3)
             assert (flags == (1 if in_shared else 0)).all(), (test, flags[:4])
 
 
