@@ -406,6 +406,14 @@ def su3_sweep(G, torch, ctx, stream):
                      "regs": G.gtr_query_variant(G.K_SU3, c)["regs"], "closed_form_ok": ok}
     G.gtr_ctx_check(ctx, stream)
     del dA, dC
+    # Fig. 11c analogue: speed-up over the LLVM 12 configuration (generic mode,
+    # coalesced globalization, no folding) of each step of the paper's ladder
+    base = res["generic_llvm12_coalesced"]["ms_per_iter"]
+    res["paper_ladder_speedup_vs_llvm12"] = {
+        "opts_disabled_simplified_globalization": base / res["generic_runtime_globalized"]["ms_per_iter"],
+        "h2s2_rtcspec_csm": base / res["csm_shared_fold"]["ms_per_iter"],
+        "h2s2_rtcspec_spmdization": base / res["spmd"]["ms_per_iter"],
+        "cuda_native": base / res["native"]["ms_per_iter"]}
     return res
 
 

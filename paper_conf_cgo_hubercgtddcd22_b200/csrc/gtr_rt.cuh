@@ -93,7 +93,9 @@ struct ThreadState {
     uint8_t nested;   // serialized nested parallel depth
     uint8_t level;    // SPMD: this thread's parallel level
     uint32_t gsp;     // global fallback stack top (words)
-    // PL_COALESCED (per warp, kept in the warp's lane states)
+};
+// PL_COALESCED only: per-lane + per-warp allocation state (after ThreadState)
+struct CoalState {
     uint32_t igsp;    // this lane's own global stack top (divergent calls)
     uint32_t frame;   // frame slot k lives in lane k: live lanes << 16 | global << 15 | words
     uint32_t wtop;    // lane 0: warp stack top in shared memory (words)
@@ -103,8 +105,15 @@ struct ThreadState {
 };
 extern __shared__ __align__(16) uint8_t g_dyn[];
 
+template <class K> __host__ __device__ constexpr uint32_t coal_offset() {
+    return (uint32_t)((K::BLOCK * sizeof(ThreadState) + 15) / 16 * 16);
+}
 template <class K> __host__ __device__ constexpr uint32_t tstate_bytes() {
-    return K::TSTATE ? (uint32_t)((K::BLOCK * sizeof(ThreadState) + 15) / 16 * 16) : 0u;
+    return coal_offset<K>() + (K::PL == 4 /*PL_COALESCED*/ ? (uint32_t)((K::BLOCK * sizeof(CoalState) + 15) / 16 * 16)
+                                                           : 0u);
+}
+template <class K> __device__ __forceinline__ CoalState &cstate() {
+    return reinterpret_cast<CoalState *>(g_dyn + coal_offset<K>())[threadIdx.x];
 }
 template <class K> __device__ __forceinline__ ThreadState &tstate() {
     return reinterpret_cast<ThreadState *>(g_dyn)[threadIdx.x];
@@ -179,8 +188,12 @@ enum class Role { Main, Worker, Exit };
 // code, guarded).
 template <class K> __device__ __forceinline__ Role team_init(const RtParams &rp) {
     if constexpr (K::TSTATE) {
-        ThreadState z = {0, 0, 0, 0, 0, 0, 0, 0, 0, 0};
+        ThreadState z = {0, 0, 0, 0};
         tstate<K>() = z;
+    }
+    if constexpr (K::PL == 4 /*PL_COALESCED*/) {
+        CoalState c = {0, 0, 0, 0, 0, 0};
+        cstate<K>() = c;
     }
     if constexpr (K::GENERIC_LIKE) {
         if ((int)threadIdx.x >= K::NT) {
@@ -360,14 +373,14 @@ template <class K> __device__ __noinline__ void free_shared(void *p, uint32_t by
 // allocate a per-lane copy from the second half of the pool (LIFO per lane).
 // `words` is the whole allocation (already x32 for a converged parallel warp);
 // `fk` returns the frame index (-1 for a per-lane copy).
-template <class K> __device__ __forceinline__ ThreadState *warp_states() {
-    return reinterpret_cast<ThreadState *>(g_dyn) + (threadIdx.x & ~31u);
+template <class K> __device__ __forceinline__ CoalState *warp_states() {
+    return reinterpret_cast<CoalState *>(g_dyn + coal_offset<K>()) + (threadIdx.x & ~31u);
 }
 template <class K> __device__ __noinline__ void *alloc_coalesced(uint32_t words, unsigned mask, int &fk) {
     const RtParams &rp = g_ts.rp;
     const uint64_t half = rp.pool_wpt / 2;
     if (mask != 0xffffffffu) {                            // divergent: per-lane copy
-        ThreadState &ts = tstate<K>();
+        CoalState &ts = cstate<K>();
         fk = -1;
         if (rp.pool != nullptr && (uint64_t)ts.igsp + words <= half) {
             uint64_t *p = rp.pool + (uint64_t)gridDim.x * K::BLOCK * half +
@@ -381,7 +394,7 @@ template <class K> __device__ __noinline__ void *alloc_coalesced(uint32_t words,
     uint64_t *p = nullptr;
     int k = -1;
     if ((threadIdx.x & 31u) == 0) {
-        ThreadState *W = warp_states<K>();
+        CoalState *W = warp_states<K>();
         const uint32_t cap = min(32u * rp.sm_stride_words, 32767u);
         const uint32_t wbase = threadIdx.x & ~31u;
         k = (int)W[0].nframes;
@@ -413,10 +426,10 @@ template <class K> __device__ __noinline__ void *alloc_coalesced(uint32_t words,
 template <class K> __device__ __noinline__ void free_coalesced(void *p, uint32_t words, int fk) {
     if (p == &g_sink_dummy) return;
     if (fk < 0) {
-        tstate<K>().igsp -= words;
+        cstate<K>().igsp -= words;
         return;
     }
-    ThreadState *W = warp_states<K>();
+    CoalState *W = warp_states<K>();
     __threadfence_block();                                // this lane's uses happen before release
     const uint32_t old = atomicSub(&W[fk].frame, 1u << 16);
     if ((old >> 16) != 1u) return;                        // other lanes still use frame fk
