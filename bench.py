@@ -355,17 +355,19 @@ def sweeps(G, torch, ctx, xs, first, seed, stream):
         fl = G.cfg(thread_limit=nt, num_teams=teams)
         row["barrier_floor_ns"] = _time(torch, stream, lambda: G.gtr_barrier_floor(ctx, fl, R, fo, stream), 2) \
             * 1e6 / R
-        # trivial body, K = 4 distinct regions, region args in static shared
-        # memory (heap-to-shared) for every mode; spmd_stack privatizes them
-        # (heap-to-stack: no guard barrier)
+        # region args in static shared memory (heap-to-shared) for every mode;
+        # spmd_stack privatizes them (heap-to-stack: no guard barrier,
+        # P:677-681).  "empty": one empty region forked R times (the runtime's
+        # own cost); "trivial_k4": 4 distinct regions with a trivial body.
         for name, m, pl in [("generic", G.GENERIC, G.PL_SHARED_STATIC),
                             ("cascade", G.GENERIC_CASCADE, G.PL_SHARED_STATIC),
                             ("csm", G.CSM, G.PL_SHARED_STATIC), ("spmd", G.SPMD, G.PL_SHARED_STATIC),
                             ("spmd_stack", G.SPMD, G.PL_STACK),
                             ("generic_runtime_nofold", G.GENERIC, G.PL_RUNTIME)]:
             c = G.cfg(m, pl, 0 if name.endswith("nofold") else 1, nt, num_teams=teams)
-            ms = _time(torch, stream, lambda: G.gtr_forkjoin(ctx, c, R, 1, 4, fo, stream), 2)
-            row[name + "_ns"] = ms * 1e6 / R
+            for tag, body, K in (("empty", 0, 1), ("trivial_k4", 1, 4)):
+                ms = _time(torch, stream, lambda: G.gtr_forkjoin(ctx, c, R, body, K, fo, stream), 2)
+                row[f"{name}_{tag}_ns"] = ms * 1e6 / R
             row[name + "_regs"] = G.gtr_query_variant(G.K_FORKJOIN, c)["regs"]
         # broadcast body (a guarded side effect producing a value): 2-barrier
         # broadcast vs the double-buffered 1-barrier form

@@ -41,16 +41,19 @@ template <class K> __device__ __forceinline__ uint64_t *acc_slots() {
     return acc;
 }
 
-template <class K, int k> struct Region {
+// BODY is a compile-time property of the program (0 empty, 1 trivial,
+// 2 broadcast) so an empty region is really empty after inlining.
+template <class K, int BODY, int k> struct Region {
     static constexpr int ID = k + 1;
     static __device__ void run(void *a) {
         const Args *x = static_cast<const Args *>(a);
-        const int body = g_p.body;
-        if (body == 1) {
+        if constexpr (BODY == 1) {
             const uint64_t t = (uint64_t)thread_num<K>();
             acc_slots<K>()[threadIdx.x] += (uint64_t)(k + 1) * (uint64_t)(x->r + 1) * (t + 1);
-        } else if (body == 2) {
+        } else if constexpr (BODY == 2) {
             acc_slots<K>()[threadIdx.x] += x->v;
+        } else {
+            (void)x;
         }
     }
 };
@@ -72,27 +75,29 @@ template <class K> struct Heavy {
     }
 };
 
-#define GTR_FJ_REGIONS(K)                                                                  \
-    Region<K, 0>, Region<K, 1>, Region<K, 2>, Region<K, 3>, Region<K, 4>, Region<K, 5>,     \
-        Region<K, 6>, Region<K, 7>, Region<K, 8>, Region<K, 9>, Region<K, 10>, Region<K, 11>, \
-        Region<K, 12>, Region<K, 13>, Region<K, 14>, Region<K, 15>
+#define GTR_FJ_REGIONS(K, B)                                                                       \
+    Region<K, B, 0>, Region<K, B, 1>, Region<K, B, 2>, Region<K, B, 3>, Region<K, B, 4>, Region<K, B, 5>, \
+        Region<K, B, 6>, Region<K, B, 7>, Region<K, B, 8>, Region<K, B, 9>, Region<K, B, 10>,              \
+        Region<K, B, 11>, Region<K, B, 12>, Region<K, B, 13>, Region<K, B, 14>, Region<K, B, 15>
 
-template <class K, int k> __device__ __forceinline__ void fork_k(int kk, void *a) {
+template <class K, int B, int k> __device__ __forceinline__ void fork_k(int kk, void *a) {
     if constexpr (k < 16) {
-        if (kk == k) parallel<K, Region<K, k>>(a);
-        else fork_k<K, k + 1>(kk, a);
+        if (kk == k) parallel<K, Region<K, B, k>>(a);
+        else fork_k<K, B, k + 1>(kk, a);
     }
 }
 
-template <class K> __device__ __forceinline__ uint64_t team_program() {
+// KMAX = 1: the team loop forks one region; KMAX = 16: region k = r mod K of
+// up to 16 distinct regions (a switch in the sequential code).
+template <class K, int BODY, int KMAX> __device__ __forceinline__ uint64_t team_program() {
     const int64_t R = g_p.R;
-    const int body = g_p.body, KK = g_p.K;
+    const int KK = g_p.K;
     const uint64_t g = (uint64_t)team_num<K>();
     uint64_t count = 0;
     int kk = 0;                                   // r mod K, kept as a counter
     for (int64_t r = 0; r < R; r++) {
         uint64_t v = 0;
-        if (body == 2)
+        if constexpr (BODY == 2)
             v = guarded_bcast<K, uint64_t>(
                 [&] {
                     unsigned long long *ctr = &g_p.out[g];
@@ -106,27 +111,33 @@ template <class K> __device__ __forceinline__ uint64_t team_program() {
             x.r = r;
             x.v = v;
         });
-        fork_k<K, 0>(kk, args.get());
-        kk = (kk + 1 == KK) ? 0 : kk + 1;
+        if constexpr (KMAX == 1) {
+            parallel<K, Region<K, BODY, 0>>(args.get());
+        } else {
+            fork_k<K, BODY, 0>(kk, args.get());
+            kk = (kk + 1 == KK) ? 0 : kk + 1;
+        }
         count += 1;
     }
     return count;
 }
 
-template <class K> __global__ void __launch_bounds__(K::BLOCK) kernel_fj(Params P, RtParams rp) {
+template <class K, int BODY, int KMAX>
+__global__ void __launch_bounds__(K::BLOCK) kernel_fj(Params P, RtParams rp) {
     const Role role = team_init<K>(rp);
     if (role == Role::Exit) return;
     acc_slots<K>()[threadIdx.x] = 0;
     if (role == Role::Worker) {
-        worker_loop<K, GTR_FJ_REGIONS(K)>();
+        if constexpr (KMAX == 1) worker_loop<K, Region<K, BODY, 0>>();
+        else worker_loop<K, GTR_FJ_REGIONS(K, BODY)>();
         return;
     }
     guarded<K>([&] { g_p = P; });
-    const uint64_t count = team_program<K>();
+    const uint64_t count = team_program<K, BODY, KMAX>();
     // all regions joined: reduce the workers' accumulators
     guarded<K>([&] {
         uint64_t res = 0;
-        if (g_p.body == 0) {
+        if constexpr (BODY == 0) {
             res = count;
         } else {
             for (int t = 0; t < K::NT; t++) res += acc_slots<K>()[t];
@@ -158,24 +169,38 @@ struct LaunchArgs {
     bool heavy;
 };
 
+template <class K, int BODY, int KMAX> int launch_fj(LaunchArgs &a) {
+    const void *fn = reinterpret_cast<const void *>(&kernel_fj<K, BODY, KMAX>);
+    Launch L;
+    int st = resolve<K>(a.ctx, a.cfg, fn, 64, &L);
+    if (st) return st;
+    if (a.info) {
+        int per_sm = 0;
+        GTR_CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, fn, K::BLOCK, L.dyn_smem));
+        return fill_info<K>(fn, L, per_sm, a.info);
+    }
+    kernel_fj<K, BODY, KMAX><<<L.teams, L.block, L.dyn_smem, a.stream>>>(a.P, L.rp);
+    GTR_CUDA_TRY(cudaGetLastError());
+    return GTR_OK;
+}
+
 template <class K> struct OpRt {
     static int run(LaunchArgs &a) {
-        const void *fn = a.heavy ? reinterpret_cast<const void *>(&kernel_heavy<K>)
-                                 : reinterpret_cast<const void *>(&kernel_fj<K>);
-        Launch L;
-        int st = resolve<K>(a.ctx, a.cfg, fn, 64, &L);
-        if (st) return st;
-        if (a.info) {
-            int per_sm = 0;
-            GTR_CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, fn, K::BLOCK, L.dyn_smem));
-            return fill_info<K>(fn, L, per_sm, a.info);
-        }
-        if (a.heavy)
+        if (a.heavy) {
+            const void *fn = reinterpret_cast<const void *>(&kernel_heavy<K>);
+            Launch L;
+            int st = resolve<K>(a.ctx, a.cfg, fn, 64, &L);
+            if (st) return st;
             kernel_heavy<K><<<L.teams, L.block, L.dyn_smem, a.stream>>>(a.P, L.rp);
-        else
-            kernel_fj<K><<<L.teams, L.block, L.dyn_smem, a.stream>>>(a.P, L.rp);
-        GTR_CUDA_TRY(cudaGetLastError());
-        return GTR_OK;
+            GTR_CUDA_TRY(cudaGetLastError());
+            return GTR_OK;
+        }
+        const bool one = a.P.K == 1;
+        switch (a.P.body) {
+        case 0: return one ? launch_fj<K, 0, 1>(a) : launch_fj<K, 0, 16>(a);
+        case 1: return one ? launch_fj<K, 1, 1>(a) : launch_fj<K, 1, 16>(a);
+        default: return one ? launch_fj<K, 2, 1>(a) : launch_fj<K, 2, 16>(a);
+        }
     }
 };
 
