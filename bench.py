@@ -319,6 +319,8 @@ def sweeps(G, torch, ctx, xs, first, seed, stream):
         for name, m in (("spmd", G.SPMD), ("csm", G.CSM), ("cascade", G.GENERIC_CASCADE),
                         ("generic", G.GENERIC)):
             variants.append((name + tag, G.cfg(m, G.PL_STACK, 1, 256, flags=sched)))
+            if not tag:     # generic modes run thread_limit + 32 threads: 128 fits more teams/SM
+                variants.append((name + "_t128", G.cfg(m, G.PL_STACK, 1, 128, flags=sched)))
     variants.insert(0, ("native_plain", G.cfg(G.NATIVE, G.PL_STACK, 1, 256)))
     for name, c in variants:
         def f():
