@@ -46,6 +46,9 @@ def lib():
         L.orc_xs_build_index_grid.restype = None
         L.orc_xs_build_index_grid.argtypes = [vp, i64, i64, vp, i64, vp]
         L.orc_grid_search.restype = i64; L.orc_grid_search.argtypes = [i64, vp, dbl]
+        L.orc_nuclide_search.restype = i64; L.orc_nuclide_search.argtypes = [vp, dbl, i64, i64]
+        L.orc_xs_build_hash_grid.restype = None
+        L.orc_xs_build_hash_grid.argtypes = [vp, i64, i64, i32, vp]
         L.orc_xs_lookup.restype = None
         L.orc_xs_lookup.argtypes = [vp, u64, u64, vp, vp, vp, vp]
         L.orc_xs_run.restype = None
@@ -73,7 +76,8 @@ class XsTables(C.Structure):
     _fields_ = [("n_iso", C.c_int64), ("n_gp", C.c_int64), ("n_union", C.c_int64),
                 ("max_num_nucs", C.c_int32),
                 ("grid", C.c_void_p), ("egrid", C.c_void_p), ("index_grid", C.c_void_p),
-                ("num_nucs", C.c_void_p), ("mats", C.c_void_p), ("concs", C.c_void_p)]
+                ("num_nucs", C.c_void_p), ("mats", C.c_void_p), ("concs", C.c_void_p),
+                ("grid_type", C.c_int32), ("hash_bins", C.c_int32), ("hash_index", C.c_void_p)]
 
 
 class RsTables(C.Structure):
@@ -114,12 +118,17 @@ def grid_search(a, q):
     return lib().orc_grid_search(len(a), _p(a), q)
 
 
+def nuclide_search(grid_n, q, low, high):
+    g = np.ascontiguousarray(grid_n, dtype=np.float64)
+    return lib().orc_nuclide_search(_p(g), q, low, high)
+
+
 # ---------------------------------------------------------------- XS
 class XsProblem:
     """Oracle-side tables: the generator's grid + the oracle's own unionized
     energy grid and index grid."""
 
-    def __init__(self, t, build_index=True):
+    def __init__(self, t, build_index=True, grid_type=0, hash_bins=10000):
         self.src = t
         self.grid = np.ascontiguousarray(t["grid"], dtype=np.float64)
         self.n_iso, self.n_gp = int(t["n_iso"]), int(t["n_gp"])
@@ -134,10 +143,16 @@ class XsProblem:
             self.index_grid = np.empty((self.n_union, self.n_iso), dtype=np.int32)
             lib().orc_xs_build_index_grid(_p(self.grid), self.n_iso, self.n_gp, _p(self.egrid),
                                           self.n_union, _p(self.index_grid))
+        self.grid_type, self.hash_bins, self.hash_index = grid_type, hash_bins, None
+        if grid_type == 2:
+            self.hash_index = np.empty((hash_bins, self.n_iso), dtype=np.int32)
+            lib().orc_xs_build_hash_grid(_p(self.grid), self.n_iso, self.n_gp, hash_bins, _p(self.hash_index))
         self.ct = XsTables(self.n_iso, self.n_gp, self.n_union, self.mats.shape[1],
                            _p(self.grid).value, _p(self.egrid).value,
                            _p(self.index_grid).value if self.index_grid is not None else None,
-                           _p(self.num_nucs).value, _p(self.mats).value, _p(self.concs).value)
+                           _p(self.num_nucs).value, _p(self.mats).value, _p(self.concs).value,
+                           grid_type, hash_bins,
+                           _p(self.hash_index).value if self.hash_index is not None else None)
 
     def lookup(self, i, seed):
         mat, am = C.c_int32(), C.c_int32()

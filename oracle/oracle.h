@@ -43,6 +43,9 @@ typedef struct {
     const int32_t *num_nucs;    /* [12]                                     */
     const int32_t *mats;        /* [12][max_num_nucs]                       */
     const double  *concs;       /* [12][max_num_nucs]                       */
+    int32_t grid_type;          /* 0 unionized, 1 nuclide, 2 hash (XSBench) */
+    int32_t hash_bins;          /* hash grid: number of energy bins         */
+    const int32_t *hash_index;  /* [hash_bins][n_iso] (grid_type 2)         */
 } orc_xs_tables;
 
 /* egrid = all n_iso*n_gp energies sorted ascending (qsort). */
@@ -52,7 +55,16 @@ void    orc_xs_build_index_grid(const double *grid, int64_t n_iso, int64_t n_gp,
                                 const double *egrid, int64_t n_union, int32_t *index_grid);
 /* lower-bound binary search of XSBench. */
 int64_t orc_grid_search(int64_t n, const double *a, double quarry);
-/* one lookup, global index i. */
+/* XSBench's per-nuclide lower-bound search in [low, high] on gridpoint
+ * energies (stride 6 doubles). */
+int64_t orc_nuclide_search(const double *grid_n, double quarry, int64_t low, int64_t high);
+/* Hash grid (XSBench): bin b starts at energy b/hash_bins; hash_index[b][n]
+ * = lower-bound index of that energy in nuclide n's grid. */
+void    orc_xs_build_hash_grid(const double *grid, int64_t n_iso, int64_t n_gp, int32_t hash_bins,
+                               int32_t *hash_index);
+/* one lookup, global index i (grid_type selects how the
+ * bracketing gridpoint of each nuclide is found: unionized index grid,
+ * per-nuclide search, or hash bin + bounded search -- all the same interval). */
 void    orc_xs_lookup(const orc_xs_tables *t, uint64_t i, uint64_t seed,
                       int32_t *mat, int64_t *u, double macro[5], int32_t *argmax);
 /* lookups [first, first+n): out[0] = hash = sum(argmax+1), out[1..12] material

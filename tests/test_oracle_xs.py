@@ -210,6 +210,44 @@ def test_hash_constructed_tables(orc, dominant, mult):
     assert out[13 + dominant] == L
 
 
+def test_nuclide_search_matches_bisect(orc):
+    rng = np.random.default_rng(4)
+    for _ in range(200):
+        n = int(rng.integers(2, 60))
+        g = np.zeros((n, 6))
+        g[:, 0] = np.sort(rng.uniform(0, 1, n))
+        lo = int(rng.integers(0, n - 1))
+        hi = int(rng.integers(lo + 1, n))
+        for q in list(rng.uniform(-0.1, 1.1, 6)) + [g[lo, 0], g[hi, 0]]:
+            # lower-bound search inside [lo, hi]: last index in [lo, hi-1] with e <= q
+            want = min(max(bisect.bisect_right(list(g[lo:hi + 1, 0]), q) - 1, 0), hi - lo - 1) + lo
+            assert orc.nuclide_search(g, q, lo, hi) == want
+
+
+def test_hash_index_closed_form(orc):
+    t = X.make_tables(7, 300, seed_t=21)
+    P = orc.XsProblem(t, grid_type=2, hash_bins=97)
+    e = t["grid"][:, :, 0]
+    for b in range(97):
+        for n in range(7):
+            cnt = np.searchsorted(e[n], b / 97.0, side="right")
+            assert P.hash_index[b, n] == min(max(cnt - 1, 0), 300 - 2)
+
+
+@pytest.mark.parametrize("n_iso,n_gp,bins", [(68, 2000, 10000), (13, 500, 37), (5, 50, 3)])
+def test_grid_types_give_identical_lookups(orc, n_iso, n_gp, bins):
+    # XSBench's three acceleration structures locate the same bracketing
+    # interval (the last gridpoint <= E, clamped), so every lookup -- and the
+    # hash -- must be identical to the unionized grid's (pinned above)
+    t = X.make_tables(n_iso, n_gp, seed_t=n_gp)
+    ref, vref = orc.XsProblem(t, grid_type=0).run(11, 3000, X.SEED_L, 2, verify=True)
+    for gt in (1, 2):
+        out, v = orc.XsProblem(t, grid_type=gt, hash_bins=bins).run(11, 3000, X.SEED_L, 2, verify=True)
+        assert np.array_equal(out, ref)
+        assert np.array_equal(v["macro"].view(np.uint64), vref["macro"].view(np.uint64))
+        assert np.array_equal(v["mat"], vref["mat"]) and np.array_equal(v["am"], vref["am"])
+
+
 def test_threads_do_not_change_results(orc):
     t = X.make_tables(68, 300)
     P = orc.XsProblem(t)
