@@ -333,6 +333,24 @@ def sweeps(G, torch, ctx, xs, first, seed, stream):
         modes[name] = {"lookups_per_s": n / (ms * 1e-3), "ms": ms, "regs": info["regs"],
                        "static_smem": info["static_smem"], "dyn_smem": info["dyn_smem"],
                        "teams_per_sm": info["teams_per_sm"], "same_result": bool(np.array_equal(r, ref))}
+    # XSBench's other acceleration structures, same lookups
+    grids = {}
+    import gtr_inputs.xs as X
+    from paper_conf_cgo_hubercgtddcd22_b200.problems import XsDevice
+    tables = X.make_tables(N_ISO, N_GP)
+    for gname, gt in (("nuclide_grid", G.XS_NUCLIDE), ("hash_grid", G.XS_HASH)):
+        xg = XsDevice(ctx, tables, grid_type=gt, hash_bins=10000)
+        for mname, c in (("spmd", G.cfg(G.SPMD, G.PL_STACK, 1, 256)),
+                         ("native_plain", G.cfg(G.NATIVE, G.PL_STACK, 1, 256))):
+            def f():
+                out.zero_()
+                G.gtr_xs_lookup(ctx, c, xg.tables, first, n, seed, out, None, stream)
+            ms = _time(torch, stream, f, 2)
+            grids[f"{gname}_{mname}"] = {"lookups_per_s": n / (ms * 1e-3), "ms": ms,
+                                         "table_bytes": xg.nbytes(),
+                                         "same_result": bool(np.array_equal(out.cpu().numpy(), ref))}
+        del xg
+    grids["unionized_spmd"] = {"lookups_per_s": modes["spmd"]["lookups_per_s"], "table_bytes": xs.nbytes()}
     # the paper's ladder (Fig. 11a) on SPMD: globalized at runtime -> h2s2 -> +fold
     ladder = {}
     for name, c in [("llvm12_coalesced", G.cfg(G.SPMD, G.PL_COALESCED, 0, 256)),
@@ -382,7 +400,7 @@ def sweeps(G, torch, ctx, xs, first, seed, stream):
             * 1e6 / R
         fj[f"thread_limit_{nt}"] = row
     G.gtr_ctx_check(ctx, stream)
-    return {"modes": modes, "ladder_spmd": ladder, "forkjoin": fj,
+    return {"modes": modes, "grid_types": grids, "ladder_spmd": ladder, "forkjoin": fj,
             "su3": su3_sweep(G, torch, ctx, stream), "rsbench": rs_sweep(G, torch, ctx, stream)}
 
 

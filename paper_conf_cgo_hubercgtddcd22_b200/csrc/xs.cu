@@ -166,10 +166,53 @@ extern "C" int gtr_xs_build_index_grid(gtr_ctx *ctx, const double *d_grid, int64
     return GTR_OK;
 }
 
+namespace gtr {
+namespace xs {
+// hash[b][n] = clamp(#{k: e_n[k] <= b * (1/bins)} - 1, 0, n_gp - 2)
+__global__ void k_hash_grid(const double *__restrict__ e, int64_t n_iso, int64_t n_gp, int32_t bins,
+                            int32_t *__restrict__ out) {
+    const int64_t total = (int64_t)bins * n_iso;
+    const double du = 1.0 / bins;
+    for (int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; t < total;
+         t += (int64_t)gridDim.x * blockDim.x) {
+        const int64_t b = t / n_iso, n = t - b * n_iso;
+        int64_t c = count_below(e + n * n_gp, n_gp, (double)b * du, true) - 1;
+        c = c < 0 ? 0 : (c > n_gp - 2 ? n_gp - 2 : c);
+        out[t] = (int32_t)c;
+    }
+}
+}  // namespace xs
+}  // namespace gtr
+
+extern "C" int gtr_xs_build_energies(gtr_ctx *ctx, const double *d_grid, int64_t n_iso, int64_t n_gp,
+                                     double *d_energies_out, void *stream) {
+    if (!ctx || !d_grid || !d_energies_out || n_iso < 1 || n_gp < 2) return GTR_EINVAL;
+    const int64_t total = n_iso * n_gp;
+    xs::k_extract_energies<<<grid_blocks(ctx, total, 256), 256, 0, static_cast<cudaStream_t>(stream)>>>(
+        d_grid, total, d_energies_out);
+    GTR_CUDA_TRY(cudaGetLastError());
+    return GTR_OK;
+}
+
+extern "C" int gtr_xs_build_hash_grid(gtr_ctx *ctx, const double *d_energies, int64_t n_iso, int64_t n_gp,
+                                      int32_t hash_bins, int32_t *d_hash_out, void *stream) {
+    if (!ctx || !d_energies || !d_hash_out || n_iso < 1 || n_gp < 2 || hash_bins < 1) return GTR_EINVAL;
+    xs::k_hash_grid<<<grid_blocks(ctx, (int64_t)hash_bins * n_iso, 256), 256, 0, static_cast<cudaStream_t>(stream)>>>(
+        d_energies, n_iso, n_gp, hash_bins, d_hash_out);
+    GTR_CUDA_TRY(cudaGetLastError());
+    return GTR_OK;
+}
+
 static bool tables_ok(const gtr_xs_tables *t) {
-    return t && t->egrid && t->index_grid && t->grid && t->num_nucs && t->mats && t->concs &&
-           t->n_iso > 0 && t->n_gp >= 2 && t->n_union >= 2 && t->n_union < (int64_t)UINT32_MAX &&
-           t->max_num_nucs > 0;
+    if (!(t && t->grid && t->num_nucs && t->mats && t->concs && t->n_iso > 0 && t->n_gp >= 2 &&
+          t->max_num_nucs > 0 && t->n_iso * t->n_gp < (int64_t)UINT32_MAX))
+        return false;
+    switch (t->grid_type) {
+    case GTR_XS_UNIONIZED: return t->egrid && t->index_grid && t->n_union >= 2;
+    case GTR_XS_NUCLIDE: return t->energies != nullptr;
+    case GTR_XS_HASH: return t->energies && t->hash_index && t->hash_bins >= 1;
+    default: return false;
+    }
 }
 
 extern "C" int gtr_xs_lookup(gtr_ctx *ctx, const gtr_launch_cfg *cfg, const gtr_xs_tables *tables,

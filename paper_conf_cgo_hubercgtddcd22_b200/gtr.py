@@ -51,7 +51,11 @@ class gtr_xs_tables(C.Structure):
     _fields_ = [("n_iso", C.c_int64), ("n_gp", C.c_int64), ("n_union", C.c_int64),
                 ("max_num_nucs", C.c_int32), ("egrid", C.c_void_p), ("index_grid", C.c_void_p),
                 ("grid", C.c_void_p), ("num_nucs", C.c_void_p), ("mats", C.c_void_p),
-                ("concs", C.c_void_p)]
+                ("concs", C.c_void_p), ("grid_type", C.c_int32), ("hash_bins", C.c_int32),
+                ("hash_index", C.c_void_p), ("energies", C.c_void_p)]
+
+
+XS_UNIONIZED, XS_NUCLIDE, XS_HASH = 0, 1, 2
 
 
 class gtr_xs_verify(C.Structure):
@@ -93,6 +97,8 @@ _proto = {
     "gtr_xs_build_workspace_bytes": (_u64, [_i64, _i64]),
     "gtr_xs_build_egrid": (_i, [_vp, _vp, _i64, _i64, _vp, _vp, _vp]),
     "gtr_xs_build_index_grid": (_i, [_vp, _vp, _i64, _i64, _vp, _vp, _vp, _vp]),
+    "gtr_xs_build_energies": (_i, [_vp, _vp, _i64, _i64, _vp, _vp]),
+    "gtr_xs_build_hash_grid": (_i, [_vp, _vp, _i64, _i64, C.c_int32, _vp, _vp]),
     "gtr_xs_lookup": (_i, [_vp, _P(gtr_launch_cfg), _P(gtr_xs_tables), _u64, _u64, _u64, _vp,
                            _P(gtr_xs_verify), _vp]),
     "gtr_xs_lookup_host": (_i, [_vp, _P(gtr_launch_cfg), _P(gtr_xs_tables), _P(gtr_xs_request), _vp, _vp]),
@@ -183,6 +189,17 @@ def gtr_xs_build_workspace_bytes(n_iso, n_gp):
 def gtr_xs_build_egrid(ctx, d_grid, n_iso, n_gp, d_egrid_out, d_workspace, stream=None):
     return _check("gtr_xs_build_egrid", _lib.gtr_xs_build_egrid(ctx, _ptr(d_grid), n_iso, n_gp, _ptr(d_egrid_out),
                                                                 _ptr(d_workspace), _stream(stream)))
+
+
+def gtr_xs_build_energies(ctx, d_grid, n_iso, n_gp, d_energies_out, stream=None):
+    return _check("gtr_xs_build_energies", _lib.gtr_xs_build_energies(ctx, _ptr(d_grid), n_iso, n_gp,
+                                                                      _ptr(d_energies_out), _stream(stream)))
+
+
+def gtr_xs_build_hash_grid(ctx, d_energies, n_iso, n_gp, hash_bins, d_hash_out, stream=None):
+    return _check("gtr_xs_build_hash_grid", _lib.gtr_xs_build_hash_grid(ctx, _ptr(d_energies), n_iso, n_gp,
+                                                                        hash_bins, _ptr(d_hash_out),
+                                                                        _stream(stream)))
 
 
 def gtr_xs_build_index_grid(ctx, d_grid, n_iso, n_gp, d_egrid, d_index_out, d_workspace, stream=None):

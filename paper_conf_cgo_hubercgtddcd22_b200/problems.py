@@ -13,31 +13,48 @@ def _dev(a, device):
 
 
 class XsDevice:
-    """XS tables on the GPU: the nuclide grid (uploaded), the unionized energy
-    grid and the index grid (built by gtr_xs_build_egrid / _index_grid)."""
+    """XS tables on the GPU: the nuclide grid (uploaded) and the acceleration
+    structure of `grid_type`, built by libgtr: unionized energy grid + index
+    grid (gtr_xs_build_egrid / _index_grid), or the compact per-nuclide
+    energies (+ the hash grid) for the nuclide / hash grid types."""
 
-    def __init__(self, ctx, t, device="cuda", stream=None):
+    def __init__(self, ctx, t, device="cuda", stream=None, grid_type=0, hash_bins=10000):
         self.n_iso, self.n_gp = int(t["n_iso"]), int(t["n_gp"])
         self.n_union = self.n_iso * self.n_gp
+        self.grid_type, self.hash_bins = grid_type, hash_bins
         self.grid = _dev(t["grid"], device)
         self.num_nucs = _dev(t["num_nucs"].astype(np.int32), device)
         self.mats = _dev(t["mats"].astype(np.int32), device)
         self.concs = _dev(t["concs"].astype(np.float64), device)
         self.max_num_nucs = int(t["mats"].shape[1])
-        self.egrid = torch.empty(self.n_union, dtype=torch.float64, device=device)
-        self.index_grid = torch.empty((self.n_union, self.n_iso), dtype=torch.int32, device=device)
-        ws = torch.empty(G.gtr_xs_build_workspace_bytes(self.n_iso, self.n_gp), dtype=torch.uint8, device=device)
-        G.gtr_xs_build_egrid(ctx, self.grid, self.n_iso, self.n_gp, self.egrid, ws, stream)
-        G.gtr_xs_build_index_grid(ctx, self.grid, self.n_iso, self.n_gp, self.egrid, self.index_grid, ws, stream)
+        self.egrid = self.index_grid = self.energies = self.hash_index = None
+        if grid_type == G.XS_UNIONIZED:
+            self.egrid = torch.empty(self.n_union, dtype=torch.float64, device=device)
+            self.index_grid = torch.empty((self.n_union, self.n_iso), dtype=torch.int32, device=device)
+            ws = torch.empty(G.gtr_xs_build_workspace_bytes(self.n_iso, self.n_gp), dtype=torch.uint8,
+                             device=device)
+            G.gtr_xs_build_egrid(ctx, self.grid, self.n_iso, self.n_gp, self.egrid, ws, stream)
+            G.gtr_xs_build_index_grid(ctx, self.grid, self.n_iso, self.n_gp, self.egrid, self.index_grid, ws,
+                                      stream)
+            del ws
+        else:
+            self.energies = torch.empty((self.n_iso, self.n_gp), dtype=torch.float64, device=device)
+            G.gtr_xs_build_energies(ctx, self.grid, self.n_iso, self.n_gp, self.energies, stream)
+            if grid_type == G.XS_HASH:
+                self.hash_index = torch.empty((hash_bins, self.n_iso), dtype=torch.int32, device=device)
+                G.gtr_xs_build_hash_grid(ctx, self.energies, self.n_iso, self.n_gp, hash_bins, self.hash_index,
+                                         stream)
         G.gtr_ctx_check(ctx, stream)           # duplicate energies -> GtrError
-        del ws
+        p = lambda x: x.data_ptr() if x is not None else None   # noqa: E731
         self.tables = G.gtr_xs_tables(self.n_iso, self.n_gp, self.n_union, self.max_num_nucs,
-                                      self.egrid.data_ptr(), self.index_grid.data_ptr(), self.grid.data_ptr(),
-                                      self.num_nucs.data_ptr(), self.mats.data_ptr(), self.concs.data_ptr())
+                                      p(self.egrid), p(self.index_grid), self.grid.data_ptr(),
+                                      self.num_nucs.data_ptr(), self.mats.data_ptr(), self.concs.data_ptr(),
+                                      grid_type, hash_bins, p(self.hash_index), p(self.energies))
 
     def nbytes(self):
         return sum(x.numel() * x.element_size() for x in
-                   (self.grid, self.egrid, self.index_grid, self.num_nucs, self.mats, self.concs))
+                   (self.grid, self.egrid, self.index_grid, self.energies, self.hash_index, self.num_nucs,
+                    self.mats, self.concs) if x is not None)
 
     def verify_buffers(self, n, device="cuda"):
         bufs = {"mat": torch.zeros(n, dtype=torch.uint8, device=device),

@@ -132,6 +132,44 @@ def test_duplicate_energies_detected(G, ctx):
         XsDevice(ctx, t)
 
 
+@pytest.fixture(scope="module", params=[1, 2], ids=["nuclide_grid", "hash_grid"])
+def dev_grid(request, G, ctx, small):
+    from paper_conf_cgo_hubercgtddcd22_b200.problems import XsDevice
+    return request.param, XsDevice(ctx, small[0], grid_type=request.param, hash_bins=10000)
+
+
+def test_hash_grid_builder_matches_oracle(G, ctx, small, orc):
+    from paper_conf_cgo_hubercgtddcd22_b200.problems import XsDevice
+    t = small[0]
+    dev = XsDevice(ctx, t, grid_type=2, hash_bins=997)
+    P = orc.XsProblem(t, build_index=False, grid_type=2, hash_bins=997)
+    assert np.array_equal(dev.hash_index.cpu().numpy(), P.hash_index)
+    assert np.array_equal(dev.energies.cpu().numpy(), t["grid"][:, :, 0])
+
+
+@pytest.mark.parametrize("variant", [(m, p, f, 256) for m in (0, 1, 2, 3) for p, f in ((3, 1), (0, 0), (4, 0))],
+                         ids=vid)
+@pytest.mark.parametrize("sched", (0, 4), ids=("bucketed", "plain"))
+def test_grid_types_bit_exact(G, ctx, dev_grid, small, variant, sched):
+    # the three grid types bracket the same gridpoints: macro XS, argmax and
+    # tallies bit-identical to the (oracle-pinned) unionized results
+    gt, dev = dev_grid
+    t, P, o_out, o_v, n = small
+    m, p, f, nt = variant
+    out, v = _run(G, ctx, dev, G.cfg(m, p, f, nt, flags=sched), 0, n)
+    assert np.array_equal(out, o_out)
+    assert np.array_equal(v["mat"], o_v["mat"]) and np.array_equal(v["am"], o_v["am"])
+    assert np.array_equal(v["macro"].view(np.uint64), o_v["macro"].view(np.uint64))
+
+
+def test_grid_types_native(G, ctx, dev_grid, small):
+    gt, dev = dev_grid
+    t, P, o_out, o_v, n = small
+    out, v = _run(G, ctx, dev, G.cfg(G.NATIVE, G.PL_STACK, 1, 256), 0, n)
+    assert np.array_equal(out, o_out)
+    assert np.array_equal(v["macro"].view(np.uint64), o_v["macro"].view(np.uint64))
+
+
 def test_variant_resources(G):
     info = G.gtr_query_variant(G.K_XS, G.cfg(G.SPMD, G.PL_STACK, 1, 256))
     assert info["block_threads"] == 256 and info["regs"] > 0 and info["num_teams"] > 0
