@@ -77,3 +77,16 @@ def test_semantics_closed_forms(orc):
     assert list(e[2 * G:]) == [7 * g + t for g in range(G) for t in range(T)]
     e = orc.sem_expected(5, G, T)
     assert list(e) == [1 + 20 + 100 + 10000 * T + 100000000 * t for g in range(G) for t in range(T)]
+    # test 6 closed forms: omp_set_num_threads(T/2+1), then a region without
+    # clause (n1 threads, nested serialized region inside), then num_threads(5)
+    e = orc.sem_expected(6, G, T)
+    n1 = T // 2 + 1
+    A, B, Cc = e[:G * T].reshape(G, T), e[G * T:G * T + 5 * G].reshape(G, 5), e[G * T + 5 * G:].reshape(G, T)
+    for g in range(G):
+        for t in range(T):
+            if t < n1:
+                assert A[g, t] == t + 1000 * n1 + 10 ** 6 + 10 ** 7 + 10 ** 8 * n1
+                assert Cc[g, t] == 20 + 100 + 1000 * t + 10 ** 7 * n1 + 10 ** 11 + 10 ** 12
+            else:
+                assert A[g, t] == 0 and Cc[g, t] == 0
+        assert list(B[g]) == [t + 5000 + 10 ** 6 for t in range(5)]
