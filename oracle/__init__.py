@@ -242,7 +242,7 @@ def fj_host_team(T, R, body, K=1):
 
 
 def sem_expected(test_id, G, T):
-    out = np.zeros(2 * G * T + 7 * G + 16, dtype=np.uint64)
+    out = np.zeros(10 * G * T + 21 * G + 16, dtype=np.uint64)
     n = lib().orc_sem_expected(test_id, G, T, _p(out), len(out))
     if n < 0:
         raise ValueError("bad semantics test id")
