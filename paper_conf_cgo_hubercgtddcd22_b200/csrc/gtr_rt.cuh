@@ -82,6 +82,9 @@ struct TeamState {
     volatile int32_t level;     // team parallel level seen by workers (generic)
     volatile int32_t nthreads;  // threads of the active parallel region
     int32_t exec_mode;          // ICV read by non-folded is_spmd()
+    volatile int32_t nvar;      // nthreads-var ICV (omp_set_num_threads)
+    uint32_t sb_count;          // software barrier of a partial-warp team:
+    volatile uint32_t sb_gen;   //   arrivals and generation
     RtParams rp;
     uint64_t bcast[2];          // guarded-value broadcast slots
 };
@@ -136,11 +139,37 @@ template <class K> __device__ __forceinline__ void team_barrier() {
 // `#pragma omp barrier` inside a parallel region: the region's threads only
 // (generic: the NT workers on named barrier 2; the main thread waits at the
 // join).  SPMD: the whole CTA.
-template <class K> __device__ __forceinline__ void omp_barrier() {
+// A team smaller than NT (num_threads clause / ICV, non-folded variants):
+// named barrier 2 over its warps when it is whole warps, else a software
+// barrier in shared memory.  Serialized nested regions: a team of one.
+static __device__ __noinline__ void soft_barrier(int n) {
+    __threadfence_block();
+    const uint32_t gen = g_ts.sb_gen;
+    if (atomicAdd(&g_ts.sb_count, 1u) == (uint32_t)n - 1u) {
+        g_ts.sb_count = 0;
+        __threadfence_block();
+        g_ts.sb_gen = gen + 1u;
+    } else {
+        while (g_ts.sb_gen == gen) __nanosleep(32);
+    }
+    __threadfence_block();
+}
+template <class K> __device__ __forceinline__ void omp_barrier_full() {
     if constexpr (K::GENERIC_LIKE)
         asm volatile("barrier.sync 2, %0;" ::"n"(K::NT) : "memory");
     else
         __syncthreads();
+}
+template <class K> __device__ __forceinline__ void omp_barrier() {
+    if constexpr (K::FOLD) {
+        omp_barrier_full<K>();
+    } else {
+        if (tstate<K>().nested) return;
+        const int n = g_ts.nthreads;
+        if (n == K::NT) omp_barrier_full<K>();
+        else if ((n & 31) == 0) asm volatile("barrier.sync 2, %0;" ::"r"(n) : "memory");
+        else soft_barrier(n);
+    }
 }
 
 // Team-wide sync of SPMD-ized sequential code (e.g. before a shared team
@@ -179,6 +208,48 @@ template <class K> __device__ __forceinline__ int num_threads() {
     else return (parallel_level<K>() == 0 || tstate<K>().nested) ? 1 : g_ts.nthreads;
 }
 
+// Thread-management ICVs and queries of nested parallelism (OpenMP 5.1
+// sec. 3.2).  Only the outermost region of a team is active:
+// nested regions are serialized, so levels >= 2 have team size 1
+// and thread number 0.  Folded variants assume what the analysis proved for
+// them: inside a parallel region of NT threads, no nesting, no
+// num_threads clause or omp_set_num_threads reaching the kernel.
+template <class K> __device__ __forceinline__ int outer_level() {          // 0 or 1
+    if constexpr (K::FOLD) return 1;
+    else if constexpr (K::MODE == SPMD) return tstate<K>().level;
+    else return threadIdx.x == K::MAIN_HW ? 0 : g_ts.level;
+}
+template <class K> __device__ __forceinline__ int active_level() {
+    if constexpr (K::FOLD) return 1;
+    else return (outer_level<K>() == 1 && g_ts.nthreads > 1) ? 1 : 0;
+}
+template <class K> __device__ __forceinline__ int max_threads() {          // omp_get_max_threads
+    if constexpr (K::FOLD) return K::NT;
+    else return min((int)g_ts.nvar, K::NT);
+}
+template <class K> __device__ __forceinline__ int ancestor_thread_num(int l) {
+    const int lev = parallel_level<K>();
+    if (l < 0 || l > lev) return -1;
+    if (l == 0) return 0;
+    if (l == 1) return (int)threadIdx.x;          // the outer (active) region
+    return 0;                                     // serialized levels
+}
+template <class K> __device__ __forceinline__ int team_size(int l) {
+    const int lev = parallel_level<K>();
+    if (l < 0 || l > lev) return -1;
+    if (l == 1) {
+        if constexpr (K::FOLD) return K::NT;
+        else return g_ts.nthreads;
+    }
+    return 1;                                     // initial team, serialized levels
+}
+// threads of the next region: the num_threads clause if given, else the
+// nthreads-var ICV; at most the team's hardware threads
+template <class K> __device__ __forceinline__ int region_threads(int clause) {
+    const int n = clause > 0 ? clause : (int)g_ts.nvar;
+    return n < K::NT ? n : K::NT;
+}
+
 // ---------------------------------------------------------------- roles
 enum class Role { Main, Worker, Exit };
 
@@ -204,6 +275,9 @@ template <class K> __device__ __forceinline__ Role team_init(const RtParams &rp)
             g_ts.level = 0;
             g_ts.nthreads = K::NT;
             g_ts.exec_mode = K::MODE;
+            g_ts.nvar = K::NT;
+            g_ts.sb_count = 0;
+            g_ts.sb_gen = 0;
             g_ts.rp = rp;
             return Role::Main;
         }
@@ -213,6 +287,9 @@ template <class K> __device__ __forceinline__ Role team_init(const RtParams &rp)
             g_ts.level = 0;
             g_ts.nthreads = K::NT;
             g_ts.exec_mode = K::MODE;
+            g_ts.nvar = K::NT;
+            g_ts.sb_count = 0;
+            g_ts.sb_gen = 0;
             g_ts.rp = rp;
         }
         __syncthreads();
@@ -222,7 +299,9 @@ template <class K> __device__ __forceinline__ Role team_init(const RtParams &rp)
 
 // ---------------------------------------------------------------- fork/join
 // Region types: struct R { static constexpr int ID = ...; static __device__ void run(void*); }
-template <class K, class R> __device__ __forceinline__ void parallel(void *args) {
+// `num_threads_clause` > 0 is the region's num_threads clause (non-folded
+// variants; threads beyond the region's team skip its body).
+template <class K, class R> __device__ __forceinline__ void parallel(void *args, int num_threads_clause = 0) {
     if constexpr (!K::FOLD) {
         if (parallel_level<K>() > 0) {          // nested: serialize
             tstate<K>().nested++;
@@ -232,9 +311,21 @@ template <class K, class R> __device__ __forceinline__ void parallel(void *args)
         }
     }
     if constexpr (K::MODE == SPMD) {
-        if constexpr (!K::FOLD) tstate<K>().level = 1;
-        R::run(args);                            // in place, all threads
-        if constexpr (!K::FOLD) tstate<K>().level = 0;
+        if constexpr (!K::FOLD) {
+            // every thread computes the same team size; publishing a changed
+            // one is a guarded side effect (its barriers only when it changes)
+            const int n = region_threads<K>(num_threads_clause);
+            if (n != g_ts.nthreads) {
+                __syncthreads();
+                if (threadIdx.x == 0) g_ts.nthreads = n;
+                __syncthreads();
+            }
+            tstate<K>().level = 1;
+            if ((int)threadIdx.x < n) R::run(args);   // in place
+            tstate<K>().level = 0;
+        } else {
+            R::run(args);                        // in place, all threads
+        }
         __syncthreads();                         // join
     } else {
         static_assert(K::GENERIC_LIKE, "parallel() needs a runtime mode");
@@ -244,6 +335,7 @@ template <class K, class R> __device__ __forceinline__ void parallel(void *args)
             g_ts.fn = &R::run;                   // address taken: GEN / CAS
         g_ts.args = args;
         g_ts.level = 1;
+        if constexpr (!K::FOLD) g_ts.nthreads = region_threads<K>(num_threads_clause);
         team_barrier<K>();                       // fork
         team_barrier<K>();                       // join
         g_ts.level = 0;
@@ -272,14 +364,21 @@ template <class K, class... Rs> __device__ void worker_loop() {
     for (;;) {
         team_barrier<K>();                       // wait for work
         void *a = g_ts.args;
+        int id = 0;
+        RegionFn fn = nullptr;
         if constexpr (K::MODE == CSM) {
-            int id = g_ts.region_id;
+            id = g_ts.region_id;
             if (id == 0) return;
-            Dispatch<K, Rs...>::csm(id, a);      // direct calls, no fallback
         } else {
-            RegionFn fn = g_ts.fn;
+            fn = g_ts.fn;
             if (fn == nullptr) return;
-            if constexpr (K::MODE == GENERIC_CASCADE) {
+        }
+        // not in this region's team (num_threads clause / ICV): straight to the join
+        const bool in_team = K::FOLD || (int)threadIdx.x < g_ts.nthreads;
+        if (in_team) {
+            if constexpr (K::MODE == CSM) {
+                Dispatch<K, Rs...>::csm(id, a);  // direct calls, no fallback
+            } else if constexpr (K::MODE == GENERIC_CASCADE) {
                 if (!Dispatch<K, Rs...>::cascade(fn, a)) fn(a);   // indirect fallback
             } else {
                 fn(a);                           // indirect call
@@ -324,6 +423,12 @@ template <class K, class T, class F> __device__ __forceinline__ T guarded_bcast(
     } else {
         return f();
     }
+}
+
+// omp_set_num_threads in the team's sequential code: a write of the team's
+// nthreads-var ICV (a guarded side effect in SPMD mode).
+template <class K> __device__ __forceinline__ void set_num_threads(int n) {
+    guarded<K>([&] { g_ts.nvar = n > 0 ? n : 1; });
 }
 
 // ---------------------------------------------------------------- globalization
@@ -586,6 +691,43 @@ template <class K, class T, class Tag, bool RO = true> struct TeamLocal {
 template <class K, class F> __device__ __forceinline__ void for_static(int64_t lo, int64_t hi, F &&body) {
     const int64_t t = thread_num<K>(), n = num_threads<K>();
     for (int64_t i = lo + t; i < hi; i += n) body(i);
+}
+
+// `for schedule(static, chunk)`: chunk k goes to thread k mod num_threads.
+template <class K, class F>
+__device__ __forceinline__ void for_static_chunk(int64_t lo, int64_t hi, int64_t chunk, F &&body) {
+    const int64_t t = thread_num<K>(), n = num_threads<K>();
+    for (int64_t c = lo + t * chunk; c < hi; c += n * chunk)
+        for (int64_t i = c; i < c + chunk && i < hi; i++) body(i);
+}
+// `for schedule(dynamic, chunk)`: threads claim chunks from a team counter
+// (zeroed by the sequential code before the region).
+template <class K, class F>
+__device__ __forceinline__ void for_dynamic(int64_t lo, int64_t hi, int64_t chunk, unsigned long long *counter,
+                                            F &&body) {
+    for (;;) {
+        const int64_t c = lo + (int64_t)atomicAdd(counter, (unsigned long long)chunk);
+        if (c >= hi) break;
+        for (int64_t i = c; i < c + chunk && i < hi; i++) body(i);
+    }
+}
+// `for schedule(guided, chunk)`: chunk = max(chunk, remaining / (2 n)),
+// claimed with compare-and-swap on a team counter (zeroed before the region).
+template <class K, class F>
+__device__ __forceinline__ void for_guided(int64_t lo, int64_t hi, int64_t chunk, unsigned long long *counter,
+                                           F &&body) {
+    const int64_t n = num_threads<K>();
+    unsigned long long cur = *reinterpret_cast<volatile unsigned long long *>(counter);
+    for (;;) {
+        const int64_t c = lo + (int64_t)cur;
+        if (c >= hi) break;
+        int64_t sz = (hi - c) / (2 * n);
+        if (sz < chunk) sz = chunk;
+        const unsigned long long seen = atomicCAS(counter, cur, cur + (unsigned long long)sz);
+        if (seen != cur) { cur = seen; continue; }
+        for (int64_t i = c; i < c + sz && i < hi; i++) body(i);
+        cur = *reinterpret_cast<volatile unsigned long long *>(counter);
+    }
 }
 
 // `for schedule(dynamic, 32)`: warps claim 32 consecutive iterations at a

@@ -61,9 +61,13 @@ SEM_VARIANTS = list(itertools.product(RUNTIME_MODES, PLACEMENTS, (0, 1), (64, 12
 def test_semantics_all_variants(G, ctx, orc, variant):
     m, p, f, nt = variant
     G_teams = 6
-    for test in range(6):
-        if test == 5 and f == 1:
-            continue                       # folding assumes no nested parallelism
+    for test in range(8):
+        if test >= 5 and f == 1:
+            # folding assumes no nesting and no thread-count ICV changes
+            with pytest.raises(G.GtrError, match="not instantiated"):
+                G.gtr_semantics(ctx, G.cfg(m, p, f, nt, num_teams=G_teams), test,
+                                torch.zeros(10 ** 5, dtype=torch.uint64, device="cuda"), 10 ** 5)
+            continue
         want = orc.sem_expected(test, G_teams, nt)
         extra = len(want) if test in (2, 3) else 0
         out = torch.zeros(len(want) + extra, dtype=torch.uint64, device="cuda")
