@@ -59,6 +59,8 @@ def lib():
         L.orc_rs_lookup.restype = None; L.orc_rs_lookup.argtypes = [vp, u64, u64, vp, vp, vp]
         L.orc_rs_run.restype = None
         L.orc_rs_run.argtypes = [vp, u64, u64, u64, C.c_int, vp, vp, vp, vp, vp]
+        L.orc_rs_work.restype = None; L.orc_rs_work.argtypes = [vp, u64, u64, u64, C.c_int, vp]
+        L.orc_rs_flops.restype = dbl; L.orc_rs_flops.argtypes = [vp, C.POINTER(dbl)]
         L.orc_fj_team.restype = u64; L.orc_fj_team.argtypes = [i32, i32, i64, i32, i32]
         L.orc_fj_host_team.restype = u64
         L.orc_fj_host_team.argtypes = [i32, i64, i32, i32, C.POINTER(dbl)]
@@ -228,6 +230,16 @@ class RsProblem:
             lib().orc_rs_run(C.byref(self.ct), first, n, seed, nthreads, _p(out),
                              None, None, None, C.byref(margin))
         return out, v, margin.value
+
+    def work(self, first, n, seed, nthreads=1):
+        """Algorithmic fp64 work of lookups [first, first+n): (counts, flops,
+        transcendentals); counts = (nuclide visits, Abrarov poles, asymptotic
+        poles).  Weights in oracle/rs.c."""
+        counts = np.zeros(3, dtype=np.uint64)
+        lib().orc_rs_work(C.byref(self.ct), first, n, seed, nthreads, _p(counts))
+        tr = C.c_double()
+        fl = lib().orc_rs_flops(_p(counts), C.byref(tr))
+        return counts, fl, tr.value
 
 
 # ---------------------------------------------------------------- fork/join

@@ -103,6 +103,16 @@ void     orc_rs_lookup(const orc_rs_tables *t, uint64_t i, uint64_t seed,
 void     orc_rs_run(const orc_rs_tables *t, uint64_t first, uint64_t n, uint64_t seed,
                     int nthreads, uint64_t out[18], uint8_t *v_mat, uint8_t *v_am,
                     double *v_macro, double *min_margin);
+/* algorithmic fp64 work (see rs.c): counts[0] nuclide visits, [1] Abrarov
+ * poles, [2] asymptotic poles (ADDED to counts); flops from the counts,
+ * *transcendentals = sin/cos/atan calls.                                   */
+#define ORC_RS_FLOPS_NUC  36.0
+#define ORC_RS_FLOPS_POLE 35.0
+#define ORC_RS_FLOPS_WA   367.0
+#define ORC_RS_FLOPS_WB   50.0
+void     orc_rs_work(const orc_rs_tables *t, uint64_t first, uint64_t n, uint64_t seed, int nthreads,
+                     uint64_t counts[3]);
+double   orc_rs_flops(const uint64_t counts[3], double *transcendentals);
 
 /* ---------------- fork/join + runtime semantics (config 2; 8(c) c6) ---- */
 /* Per-team results of the fork/join program with T workers and R regions.

@@ -37,7 +37,7 @@ int gtr_internal_query_sem(gtr_ctx *ctx, const gtr_launch_cfg *cfg, gtr_variant_
 
 extern "C" int gtr_semantics(gtr_ctx *ctx, const gtr_launch_cfg *cfg, int32_t test_id, uint64_t *d_out,
                              int64_t out_len, void *stream) {
-    if (!ctx || !cfg || !d_out || test_id < 0 || test_id > 7 || out_len < 0) return GTR_EINVAL;
+    if (!ctx || !cfg || !d_out || test_id < 0 || test_id > 8 || out_len < 0) return GTR_EINVAL;
     sem::Params P;
     P.test = test_id;
     P.T = cfg->thread_limit;

@@ -61,7 +61,7 @@ SEM_VARIANTS = list(itertools.product(RUNTIME_MODES, PLACEMENTS, (0, 1), (64, 12
 def test_semantics_all_variants(G, ctx, orc, variant):
     m, p, f, nt = variant
     G_teams = 6
-    for test in range(8):
+    for test in range(9):
         if test >= 5 and f == 1:
             # folding assumes no nesting and no thread-count ICV changes
             with pytest.raises(G.GtrError, match="not instantiated"):

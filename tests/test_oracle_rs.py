@@ -135,3 +135,40 @@ def test_rs_generator_structure():
         nw = int(t["n_windows"][n])
         assert w["start"][n, 0] == 0
         assert w["end"][n, nw - 1] == t["n_poles"][n] - 1
+
+
+# ---------------------------------------------------------------- work counts
+def test_rs_work_counts_brute_force(orc, rs_small):
+    """orc_rs_work (the algorithmic-flop counter of SURVEY 8(d) config 4)
+    equals a direct walk of the lookups: nuclide visits, and poles per
+    Faddeeva branch (|Z| < 6 or not); flops follow the documented weights."""
+    import math
+    t = rs_small
+    first, n = 17, 150
+    vis = ab = asy = 0
+    for i in range(first, first + n):
+        E, s = orc.lcg_double(orc.lcg_ff(X.SEED_L, 2 * i))
+        mat, _ = orc.pick_mat(s)
+        for j in range(int(t["num_nucs"][mat])):
+            nuc = int(t["mats"][mat, j])
+            nw = int(t["n_windows"][nuc])
+            w = int(E / (1.0 / nw))
+            w = nw - 1 if w == nw else w
+            vis += 1
+            for p in range(int(t["windows"]["start"][nuc, w]), int(t["windows"]["end"][nuc, w])):
+                ea = t["poles"]["EA"][nuc, p]
+                zr, zi = (E - ea[0]) * 0.5, (0.0 - ea[1]) * 0.5
+                if math.sqrt(zr * zr + zi * zi) < 6.0:
+                    ab += 1
+                else:
+                    asy += 1
+    P = orc.RsProblem(t)
+    counts, flops, trans = P.work(first, n, X.SEED_L)
+    assert list(P.work(first, n, X.SEED_L, 4)[0]) == list(counts)
+    assert list(counts) == [vis, ab, asy]
+    assert vis > 0 and ab > 0
+    assert flops == 36 * vis + (35 + 367) * ab + (35 + 50) * asy
+    assert trans == 11 * vis + 2 * ab
+    # visits also equal sum over the material tallies of num_nucs
+    out, _, _ = P.run(first, n, X.SEED_L)
+    assert vis == int((out[1:13].astype(np.int64) * t["num_nucs"].astype(np.int64)).sum())

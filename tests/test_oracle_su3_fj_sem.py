@@ -92,13 +92,14 @@ def test_semantics_closed_forms(orc):
         assert list(B[g]) == [t + 5000 + 10 ** 6 for t in range(5)]
 
 
+@pytest.mark.parametrize("test", [7, 8])
 @pytest.mark.parametrize("T", [32, 64, 128])
-def test_semantics_schedules_closed_forms(orc, T):
+def test_semantics_schedules_closed_forms(orc, T, test):
     """test 7: static chunks dealt round robin (chunk k -> thread k mod n,
     OpenMP 5.1 sec. 2.11.4); dynamic and guided run each iteration once."""
     G = 3
-    L, n = 3 * T + 7, T // 2 + 1
-    e = orc.sem_expected(7, G, T)
+    L, n = 3 * T + 7, (T // 2 + 1 if test == 7 else T // 2)
+    e = orc.sem_expected(test, G, T)
     assert len(e) == 3 * G * L + G * T
     own, dyn, gui, chk = (e[:G * L].reshape(G, L), e[G * L:2 * G * L].reshape(G, L),
                           e[2 * G * L:3 * G * L].reshape(G, L), e[3 * G * L:].reshape(G, T))
