@@ -236,8 +236,10 @@ def run_gtr(a):
             traffic, traffic_src = ks[0]["dram_bytes_per_launch"], os.path.relpath(profs[-1], ROOT)
 
     extra = {}
+    if not a.no_sweep:      # 180 GB HBM: the XS tables stay resident
+        extra["sharded"] = sharded_apps(G, torch, ctx, rank, ws, dist, stream, dev)
     if rank == 0 and not a.no_sweep:
-        extra = sweeps(G, torch, ctx, xs, first, seed, stream)
+        extra.update(sweeps(G, torch, ctx, xs, first, seed, stream))
 
     # e2e through the public host-buffer entry point (H2D request, D2H results)
     h_out = torch.zeros(18, dtype=torch.uint64).pin_memory()
@@ -439,15 +441,99 @@ def su3_sweep(G, torch, ctx, stream):
     return res
 
 
-def rs_sweep(G, torch, ctx, stream, n=2_000_000):
-    """Config 4: RSBench multipole lookups (355 nuclides), lookups/s per mode
-    on the first n of the 10M lookups."""
+def fp64_peak(G, torch, ctx, stream):
+    """Measured fp64 FMA ceiling (gtr_fp64_probe), TFLOP/s."""
+    scratch = torch.zeros(1, dtype=torch.uint64, device="cuda")
+    fl = G.gtr_fp64_probe(ctx, 4096, scratch, stream)
+    ms = _time(torch, stream, lambda: G.gtr_fp64_probe(ctx, 4096, scratch, stream), 5)
+    return fl / (ms * 1e-3) / 1e12
+
+
+def rs_roofline(G, torch, ctx, stream, first, n, ms):
+    """`bound: alu` roofline of the RS lookup kernel: algorithmic flops of the
+    timed lookups (profiles/rs_work.json, written by tools/rs_work.py from the
+    oracle's work counter) per second vs the measured fp64 FMA ceiling."""
+    p = os.path.join(ROOT, "profiles", "rs_work.json")
+    if not os.path.exists(p):
+        return None
+    w = json.load(open(p))
+    if (w["first"], w["n"]) != (first, n):
+        return None
+    peak = fp64_peak(G, torch, ctx, stream)
+    ach = w["flops"] / (ms * 1e-3) / 1e12
+    return {"bound": "alu", "achieved": ach, "peak": peak, "unit": "TFLOP/s", "frac": ach / peak,
+            "traffic": None, "flops_per_launch": w["flops"], "transcendentals_per_launch": w["transcendentals"],
+            "peak_source": "measured: gtr_fp64_probe (independent DFMA chains, 2 flops each); nominal "
+                           "148 SM x 64 fp64 lanes x 2 x 1.965 GHz = 37.2 TFLOP/s",
+            "flops_source": "profiles/rs_work.json (oracle work counter, tools/rs_work.py)"}
+
+
+def sharded_apps(G, torch, ctx, rank, ws, dist, stream, dev):
+    """RSBench lookups and SU3 sites sharded over the ranks
+    (weak scaling), timed on the device, max over ranks.  RS: 10M lookups per
+    GPU + the same NCCL all-reduce of the 18 u64 results as XS.  SU3: 32^4
+    sites per GPU (A, C sharded, B replicated), no collective on the data path;
+    the closed form (C == 1 exactly) is checked on every rank."""
+    import gtr_inputs.rs as RS
+    import gtr_inputs.su3 as S
+    import gtr_inputs.xs as X
+    from paper_conf_cgo_hubercgtddcd22_b200.problems import RsDevice, su3_device
+    from paper_conf_cgo_hubercgtddcd22_b200.dist import shard_range, site_shard, combine_results, max_over_ranks
+    res = {}
+    n_rs = 10_000_000
+    first, n = shard_range(rank, ws, n_rs)
+    rsd = RsDevice(RS.make_tables(), device=dev)
+    out = torch.zeros(18, dtype=torch.uint64, device=dev)
+    c = G.cfg(G.SPMD, G.PL_STACK, 1, 128)
+
+    def rs_step():
+        out.zero_()
+        G.gtr_rs_lookup(ctx, c, rsd.tables, first, n, X.SEED_L, out, None, stream)
+
+    ms = _time(torch, stream, rs_step, 2)
+    t = torch.tensor([ms], dtype=torch.float64, device=dev)
+    if dist is not None:
+        combine_results(out)
+        max_over_ranks(t)
+    ms = float(t[0])
+    r = out.cpu().numpy()
+    res["rsbench"] = {"workload": f"{n_rs} lookups per GPU (global ids [r*{n_rs}, (r+1)*{n_rs})), "
+                                  "SPMD + heap-to-stack + folding, thread_limit 128",
+                      "n_gpus": ws, "lookups_per_s": ws * n / (ms * 1e-3), "ms_max_over_ranks": ms,
+                      "hash": int(r[0]), "collective": "NCCL all_reduce(SUM) of 18 u64" if ws > 1 else None}
+    del rsd
+    sites = 32 ** 4
+    f0, m = site_shard(rank, ws, sites)
+    A, B = S.make_lattice(m, "constant", first_site=f0)
+    dA, dB = su3_device(A, B, device=dev)
+    del A
+    dC = torch.empty_like(dA)
+    for name, cc in (("native", G.cfg(G.NATIVE, G.PL_STACK, 1, 256)), ("spmd", G.cfg(G.SPMD, G.PL_STACK, 1, 64))):
+        ms = _time(torch, stream, lambda: G.gtr_su3_mat_nn(ctx, cc, dA, dB, dC, m, 1, stream), 3)
+        ok = bool(torch.all(dC.view(-1, 2)[:, 0] == 1.0).item()) and bool(torch.all(dC.view(-1, 2)[:, 1] == 0.0).item())
+        t = torch.tensor([ms, 0.0 if ok else 1.0], dtype=torch.float64, device=dev)
+        if dist is not None:
+            max_over_ranks(t)
+        ms = float(t[0])
+        res[f"su3_{name}"] = {"workload": "32^4 sites per GPU, constant inputs", "n_gpus": ws,
+                              "ms_per_iter_max_over_ranks": ms, "sites_per_s": ws * m / (ms * 1e-3),
+                              "gb_s_aggregate": ws * m * 1152 / (ms * 1e-3) / 1e9,
+                              "closed_form_ok_all_ranks": float(t[1]) == 0.0}
+    del dA, dC
+    G.gtr_ctx_check(ctx, stream)
+    torch.cuda.empty_cache()
+    return res
+
+
+def rs_sweep(G, torch, ctx, stream, n=10_000_000):
+    """Config 4: RSBench multipole lookups (355 nuclides, 10M lookups),
+    lookups/s per mode."""
     import gtr_inputs.rs as RS
     import gtr_inputs.xs as X
     from paper_conf_cgo_hubercgtddcd22_b200.problems import RsDevice
     dev = RsDevice(RS.make_tables())
     out = torch.zeros(18, dtype=torch.uint64, device="cuda")
-    res = {"workload": f"355 nuclides, ~1000 poles / 100 windows each, first {n} of 10M lookups"}
+    res = {"workload": f"355 nuclides, ~1000 poles / 100 windows each, {n} lookups"}
     ref = None
     for name, c in [("native_plain", G.cfg(G.NATIVE, G.PL_STACK, 1, 128)),
                     ("spmd", G.cfg(G.SPMD, G.PL_STACK, 1, 128)),
@@ -466,6 +552,7 @@ def rs_sweep(G, torch, ctx, stream, n=2_000_000):
         res[name] = {"lookups_per_s": n / (ms * 1e-3), "ms": ms, "regs": G.gtr_query_variant(G.K_RS, c)["regs"],
                      "same_result": bool(np.array_equal(r, ref))}
     G.gtr_ctx_check(ctx, stream)
+    res["roofline_spmd"] = rs_roofline(G, torch, ctx, stream, 0, n, res["spmd"]["ms"])
     return res
 
 

@@ -46,6 +46,11 @@ def lcg_states(seed, n):
     return out
 
 
-def uniform(seed, n):
-    """n draws U = s / 2^63 in [0, 1) (u64 -> f64 rounds to nearest, /2^63 exact)."""
+def uniform(seed, n, skip=0):
+    """n draws U = s / 2^63 in [0, 1) (u64 -> f64 rounds to nearest, /2^63 exact),
+    starting after the first `skip` draws of the stream (shards of a global
+    input)."""
+    if skip:
+        a_s, c_s = _jump(skip)
+        seed = (a_s * seed + c_s) & MASK63
     return lcg_states(seed, n).astype(np.float64) / float(1 << 63)

@@ -22,8 +22,8 @@ def lattice_sites(L):
     return L ** 4
 
 
-def _random_su3(n, seed):
-    u = uniform(seed, n * 12).reshape(n, 2, 3, 2) * 2.0 - 1.0
+def _random_su3(n, seed, skip=0):
+    u = uniform(seed, n * 12, skip=skip * 12).reshape(n, 2, 3, 2) * 2.0 - 1.0
     v1 = u[:, 0, :, 0] + 1j * u[:, 0, :, 1]
     v2 = u[:, 1, :, 0] + 1j * u[:, 1, :, 1]
     v1 = v1 / np.linalg.norm(v1, axis=1, keepdims=True)
@@ -33,14 +33,16 @@ def _random_su3(n, seed):
     return np.stack([v1, v2, v3], axis=1)          # rows are orthonormal
 
 
-def make_lattice(sites, kind="random", seed=SEED_SU3):
-    """Return (A, B) as complex128 arrays [sites,4,3,3] and [4,3,3]."""
+def make_lattice(sites, kind="random", seed=SEED_SU3, first_site=0):
+    """Return (A, B) as complex128 arrays [sites,4,3,3] and [4,3,3]: sites
+    [first_site, first_site + sites) of the global lattice (a rank's shard;
+    B is replicated)."""
     if kind == "constant":
         A = np.ones((sites, 4, 3, 3), dtype=np.complex128)
         B = np.full((4, 3, 3), 1.0 / 3.0, dtype=np.complex128)
         return A, B
     if kind != "random":
         raise ValueError(kind)
-    A = _random_su3(sites * 4, seed).reshape(sites, 4, 3, 3)
+    A = _random_su3(sites * 4, seed, skip=first_site * 4).reshape(sites, 4, 3, 3)
     B = _random_su3(4, seed + 1).reshape(4, 3, 3)
     return np.ascontiguousarray(A), np.ascontiguousarray(B)

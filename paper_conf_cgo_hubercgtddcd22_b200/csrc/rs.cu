@@ -96,3 +96,37 @@ extern "C" int gtr_rs_lookup(gtr_ctx *ctx, const gtr_launch_cfg *cfg, const gtr_
                      nullptr};
     return rs::launch(a);
 }
+
+// ---------------------------------------------------------------- fp64 probe
+// The fp64 ALU ceiling of the RS roofline, measured: every thread runs 8
+// independent chains of `iters` DFMA (a = a*b + c, 2 flops each), 8 warps x
+// 4 CTAs per SM.  d_out[0] receives a data-dependent sum (keeps the chains).
+namespace gtr {
+namespace rs {
+__global__ void __launch_bounds__(256) kernel_fp64_probe(int64_t iters, double b, double c,
+                                                         unsigned long long *out) {
+    double a[8];
+#pragma unroll
+    for (int k = 0; k < 8; k++) a[k] = (double)(threadIdx.x + k) * 1e-3;
+    for (int64_t i = 0; i < iters; i++) {
+#pragma unroll
+        for (int k = 0; k < 8; k++) a[k] = __fma_rn(a[k], b, c);
+    }
+    double s = 0.0;
+#pragma unroll
+    for (int k = 0; k < 8; k++) s += a[k];
+    if (s == 12345.678) atomicAdd(out, 1ull);             // never true; keeps the work
+}
+}  // namespace rs
+}  // namespace gtr
+
+extern "C" int gtr_fp64_probe(gtr_ctx *ctx, int64_t iters, uint64_t *d_out, double *flops_per_launch,
+                              void *stream) {
+    if (!ctx || !d_out || iters < 1) return GTR_EINVAL;
+    const int blocks = 4 * ctx->num_sms;
+    rs::kernel_fp64_probe<<<blocks, 256, 0, static_cast<cudaStream_t>(stream)>>>(
+        iters, 0.999999, 1e-7, reinterpret_cast<unsigned long long *>(d_out));
+    GTR_CUDA_TRY(cudaGetLastError());
+    if (flops_per_launch) *flops_per_launch = 2.0 * 8.0 * (double)iters * 256.0 * (double)blocks;
+    return GTR_OK;
+}

@@ -1,4 +1,5 @@
-"""Multi-GPU plumbing for the sharded lookups.
+"""Multi-GPU plumbing for the sharded lookups and lattices (SURVEY.md 8(e),
+NEXT f1).
 
 Lookups are independent and defined by their global id, so the N > 1 path is
 a partition of the id range plus one all-reduce of the 18 u64 results (hash +
@@ -42,3 +43,19 @@ def max_over_ranks(values, group=None):
     import torch.distributed as dist
     dist.all_reduce(values, op=dist.ReduceOp.MAX, group=group)
     return values
+
+
+def site_shard(rank, world_size, sites_per_rank):
+    """SU3 weak scaling: rank r owns lattice sites [r*S, (r+1)*S) of A and C;
+    B (4 links) is replicated.  Sites are independent: no collective on the
+    data path."""
+    return shard_range(rank, world_size, sites_per_rank)
+
+
+def gather_shards(local, group=None):
+    """Concatenate every rank's shard along dim 0 (validation only -- the
+    shards stay resident on their GPUs in the benchmark)."""
+    import torch.distributed as dist
+    parts = [torch.empty_like(local) for _ in range(dist.get_world_size(group))]
+    dist.all_gather(parts, local.contiguous(), group=group)
+    return torch.cat(parts, 0)

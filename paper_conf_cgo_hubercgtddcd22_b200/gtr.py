@@ -93,6 +93,7 @@ _proto = {
     "gtr_query_variant": (_i, [_i, _P(gtr_launch_cfg), _P(gtr_variant_info)]),
     "gtr_forkjoin": (_i, [_vp, _P(gtr_launch_cfg), _i64, C.c_int32, C.c_int32, _vp, _vp]),
     "gtr_barrier_floor": (_i, [_vp, _P(gtr_launch_cfg), _i64, _vp, _vp]),
+    "gtr_fp64_probe": (_i, [_vp, _i64, _vp, _P(C.c_double), _vp]),
     "gtr_semantics": (_i, [_vp, _P(gtr_launch_cfg), C.c_int32, _vp, _i64, _vp]),
     "gtr_xs_build_workspace_bytes": (_u64, [_i64, _i64]),
     "gtr_xs_build_egrid": (_i, [_vp, _vp, _i64, _i64, _vp, _vp, _vp]),
@@ -175,6 +176,13 @@ def gtr_forkjoin(ctx, launch_cfg, regions, body, n_distinct, d_out, stream=None)
 def gtr_barrier_floor(ctx, launch_cfg, iters, d_out, stream=None):
     return _check("gtr_barrier_floor", _lib.gtr_barrier_floor(ctx, C.byref(launch_cfg), iters, _ptr(d_out),
                                                               _stream(stream)))
+
+
+def gtr_fp64_probe(ctx, iters, d_out, stream=None):
+    """Launch the fp64 FMA probe; returns the flops of one launch."""
+    f = C.c_double()
+    _check("gtr_fp64_probe", _lib.gtr_fp64_probe(ctx, iters, _ptr(d_out), C.byref(f), _stream(stream)))
+    return f.value
 
 
 def gtr_semantics(ctx, launch_cfg, test_id, d_out, out_len, stream=None):

@@ -74,3 +74,48 @@ def test_u64_wraparound_through_int64_view():
     a = torch.tensor([2 ** 63 + 5], dtype=torch.uint64)
     v = a.view(torch.int64)
     assert v.view(torch.uint64)[0] == a[0]
+
+
+def _worker_apps(rank, ws, port, q):
+    """RS lookups and SU3 sites sharded over ranks."""
+    import torch.distributed as dist
+    import oracle
+    import gtr_inputs.rs as RS
+    import gtr_inputs.su3 as S
+    from paper_conf_cgo_hubercgtddcd22_b200.dist import shard_range, site_shard, combine_results, gather_shards
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=ws)
+    t = RS.make_tables(n_nuc=20, avg_poles=60, avg_windows=6)
+    first, n = shard_range(rank, ws, 40)
+    out_np, _, _ = oracle.RsProblem(t).run(first, n, X.SEED_L, 1)
+    rs = torch.from_numpy(out_np.copy())
+    combine_results(rs)
+    f, m = site_shard(rank, ws, 7)
+    A, B = S.make_lattice(m, "random", first_site=f)       # this rank's shard only
+    Cl = torch.from_numpy(oracle.su3_mat_nn(A, B).view(np.float64).copy())
+    Cg = gather_shards(Cl)
+    if rank == 0:
+        q.put((rs.numpy().copy(), Cg.numpy().copy()))
+    dist.destroy_process_group()
+
+
+@pytest.mark.parametrize("ws", [2, 3])
+def test_sharded_rs_and_su3_equal_global(orc, ws):
+    import gtr_inputs.rs as RS
+    import gtr_inputs.su3 as S
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_worker_apps, args=(r, ws, port, q)) for r in range(ws)]
+    for p in procs:
+        p.start()
+    rs, Cg = q.get(timeout=180)
+    for p in procs:
+        p.join(timeout=120)
+        assert p.exitcode == 0
+    t = RS.make_tables(n_nuc=20, avg_poles=60, avg_windows=6)
+    want, _, _ = orc.RsProblem(t).run(0, 40 * ws, X.SEED_L, 1)
+    assert np.array_equal(rs, want)
+    A, B = S.make_lattice(7 * ws, "random")                 # the global lattice
+    assert np.array_equal(Cg, orc.su3_mat_nn(A, B).view(np.float64))
