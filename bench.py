@@ -353,6 +353,27 @@ def sweeps(G, torch, ctx, xs, first, seed, stream):
                                          "same_result": bool(np.array_equal(out.cpu().numpy(), ref))}
         del xg
     grids["unionized_spmd"] = {"lookups_per_s": modes["spmd"]["lookups_per_s"], "table_bytes": xs.nbytes()}
+    # XSBench's history-based mode and sorted event-based variant (SURVEY NEXT
+    # f2): same lookups, same results; the sorted step includes its sampling
+    # pass and counting sort
+    f2 = {}
+    ws = torch.empty(G.gtr_xs_sorted_workspace_bytes(n), dtype=torch.uint8, device="cuda")
+    for name, c, sorted_ in [("spmd_history", G.cfg(G.SPMD, G.PL_STACK, 1, 256, flags=G.F_HISTORY), False),
+                             ("native_history", G.cfg(G.NATIVE, G.PL_STACK, 1, 256, flags=G.F_HISTORY), False),
+                             ("spmd_sorted", G.cfg(G.SPMD, G.PL_STACK, 1, 256), True),
+                             ("csm_sorted", G.cfg(G.CSM, G.PL_STACK, 1, 256), True),
+                             ("generic_sorted", G.cfg(G.GENERIC, G.PL_STACK, 1, 256), True),
+                             ("native_sorted", G.cfg(G.NATIVE, G.PL_STACK, 1, 256), True)]:
+        def f():
+            out.zero_()
+            if sorted_:
+                G.gtr_xs_lookup_sorted(ctx, c, xs.tables, first, n, seed, out, ws, None, stream)
+            else:
+                G.gtr_xs_lookup(ctx, c, xs.tables, first, n, seed, out, None, stream)
+        ms = _time(torch, stream, f, 3)
+        f2[name] = {"lookups_per_s": n / (ms * 1e-3), "ms": ms,
+                    "same_result": bool(np.array_equal(out.cpu().numpy(), ref))}
+    del ws
     # the paper's ladder (Fig. 11a) on SPMD: globalized at runtime -> h2s2 -> +fold
     ladder = {}
     for name, c in [("llvm12_coalesced", G.cfg(G.SPMD, G.PL_COALESCED, 0, 256)),
@@ -402,7 +423,7 @@ def sweeps(G, torch, ctx, xs, first, seed, stream):
             * 1e6 / R
         fj[f"thread_limit_{nt}"] = row
     G.gtr_ctx_check(ctx, stream)
-    return {"modes": modes, "grid_types": grids, "ladder_spmd": ladder, "forkjoin": fj,
+    return {"modes": modes, "grid_types": grids, "history_and_sorted": f2, "ladder_spmd": ladder, "forkjoin": fj,
             "su3": su3_sweep(G, torch, ctx, stream), "rsbench": rs_sweep(G, torch, ctx, stream)}
 
 

@@ -18,8 +18,18 @@ template <int NT> __global__ void __launch_bounds__(NT) kernel_native(Params P) 
     if (P.req) { P.first = P.req->first; P.n = P.req->n; P.seed = P.req->seed; }
     __syncthreads();
     const uint64_t stride = (uint64_t)gridDim.x * NT;
-    for (uint64_t k = (uint64_t)blockIdx.x * NT + threadIdx.x; k < P.n; k += stride)
-        lookup<KN>(P, P.first + k, tally);
+    if (P.s_perm) {                                   // sorted mode: thread per sorted position
+        for (uint64_t q = (uint64_t)blockIdx.x * NT + threadIdx.x; q < P.n; q += stride)
+            lookup_sorted<KN>(P, q, tally);
+    } else if (P.history) {                           // history mode: thread per particle
+        const uint64_t np = (P.n + kHistoryLookups - 1) / kHistoryLookups;
+        for (uint64_t p = (uint64_t)blockIdx.x * NT + threadIdx.x; p < np; p += stride)
+            for (uint64_t k = p * kHistoryLookups; k < P.n && k < (p + 1) * kHistoryLookups; k++)
+                lookup<KN>(P, P.first + k, tally);
+    } else {
+        for (uint64_t k = (uint64_t)blockIdx.x * NT + threadIdx.x; k < P.n; k += stride)
+            lookup<KN>(P, P.first + k, tally);
+    }
     __syncthreads();
     flush(tally, P.out, threadIdx.x, NT);
 }
@@ -105,6 +115,7 @@ inline int launch(LaunchArgs &a) {
     const gtr_launch_cfg *c = a.cfg;
     if (!valid_cfg(c)) return GTR_EINVAL;
     a.P.plain = (c->flags & GTR_F_PLAIN) ? 1 : 0;
+    a.P.history = (c->flags & GTR_F_HISTORY) ? 1 : 0;
     if (c->mode == NATIVE) {
         if (c->thread_limit == 128) return run_native<128>(a);
         if (c->thread_limit == 256) return run_native<256>(a);
@@ -241,4 +252,106 @@ extern "C" int gtr_xs_lookup_host(gtr_ctx *ctx, const gtr_launch_cfg *cfg, const
     GTR_CUDA_TRY(cudaMemcpyAsync(h_out, d_out, 18 * sizeof(uint64_t), cudaMemcpyDeviceToHost, s));
     GTR_CUDA_TRY(cudaStreamSynchronize(s));
     return GTR_OK;
+}
+
+// ---------------------------------------------------------------- sorted mode
+// XSBench's sorted event-based variant: sample every lookup,
+// counting-sort the lookups by (material, energy bucket), then run them in
+// that order -- neighbouring threads share a material (equal-length nuclide
+// loops) and nearly equal energies (the same gridpoints, adjacent index-grid
+// rows).  Results are identical: each lookup's arithmetic is its own, the
+// tallies are sums.  Workspace (caller-owned, gtr_xs_sorted_workspace_bytes):
+//   key[n] u32 | mu[n] u32 (unsorted) | perm[n] u32 | smu[n] u32 | hist[12*NB] u32 | totals[256] u32
+namespace gtr {
+namespace xs {
+constexpr uint32_t kSortBuckets = 1u << 14;           // energy buckets per material
+constexpr uint32_t kSortBins = 12u * kSortBuckets;
+
+__global__ void k_sort_sample(Params P, uint32_t *__restrict__ key, uint32_t *__restrict__ mu,
+                              uint32_t *__restrict__ hist) {
+    using KN = Cfg<NATIVE, PL_STACK, true, 128>;
+    for (uint64_t k = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; k < P.n;
+         k += (uint64_t)gridDim.x * blockDim.x) {
+        double E;
+        int mat;
+        int64_t u;
+        sample<KN>(P, P.first + k, E, mat, u);
+        uint32_t eb = (uint32_t)(E * (double)kSortBuckets);
+        eb = eb < kSortBuckets ? eb : kSortBuckets - 1;
+        const uint32_t kk = (uint32_t)mat * kSortBuckets + eb;
+        key[k] = kk;
+        mu[k] = ((uint32_t)mat << 28) | (uint32_t)u;
+        atomicAdd(hist + kk, 1u);
+    }
+}
+// exclusive scan of hist[kSortBins] in place: per 1024-bin block a shared-
+// memory scan + the block total, then every block adds the totals before it
+constexpr uint32_t kScanBlocks = kSortBins / 1024;
+__global__ void __launch_bounds__(1024) k_sort_scan_local(uint32_t *hist, uint32_t *totals) {
+    __shared__ uint32_t part[1024];
+    uint32_t *h = hist + (size_t)blockIdx.x * 1024;
+    const uint32_t x = h[threadIdx.x];
+    part[threadIdx.x] = x;
+    __syncthreads();
+    for (uint32_t off = 1; off < 1024; off <<= 1) {       // Hillis-Steele inclusive scan
+        const uint32_t v = threadIdx.x >= off ? part[threadIdx.x - off] : 0u;
+        __syncthreads();
+        part[threadIdx.x] += v;
+        __syncthreads();
+    }
+    h[threadIdx.x] = part[threadIdx.x] - x;
+    if (threadIdx.x == 1023) totals[blockIdx.x] = part[1023];
+}
+__global__ void __launch_bounds__(1024) k_sort_scan_add(uint32_t *hist, const uint32_t *totals) {
+    __shared__ uint32_t off;
+    if (threadIdx.x < 32) {
+        uint32_t s = 0;
+        for (uint32_t b = threadIdx.x; b < blockIdx.x; b += 32) s += totals[b];
+        for (int o = 16; o > 0; o >>= 1) s += __shfl_xor_sync(0xffffffffu, s, o);
+        if (threadIdx.x == 0) off = s;
+    }
+    __syncthreads();
+    hist[(size_t)blockIdx.x * 1024 + threadIdx.x] += off;
+}
+__global__ void k_sort_scatter(uint64_t n, const uint32_t *__restrict__ key, const uint32_t *__restrict__ mu,
+                               uint32_t *__restrict__ cursor, uint32_t *__restrict__ perm,
+                               uint32_t *__restrict__ smu) {
+    for (uint64_t k = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; k < n; k += (uint64_t)gridDim.x * blockDim.x) {
+        const uint32_t pos = atomicAdd(cursor + key[k], 1u);
+        perm[pos] = (uint32_t)k;
+        smu[pos] = mu[k];
+    }
+}
+static_assert(kSortBins % 1024 == 0 && kScanBlocks <= 256, "scan split");
+}  // namespace xs
+}  // namespace gtr
+
+extern "C" uint64_t gtr_xs_sorted_workspace_bytes(uint64_t n) {
+    return 16u * n + 4u * (uint64_t)(xs::kSortBins + 256);
+}
+
+extern "C" int gtr_xs_lookup_sorted(gtr_ctx *ctx, const gtr_launch_cfg *cfg, const gtr_xs_tables *tables,
+                                    uint64_t first, uint64_t n, uint64_t seed, uint64_t *d_out,
+                                    const gtr_xs_verify *verify, void *d_workspace, uint64_t workspace_bytes,
+                                    void *stream) {
+    if (!ctx || !cfg || !tables_ok(tables) || !d_out || !d_workspace) return GTR_EINVAL;
+    if (n == 0) return GTR_OK;
+    if (n > 0xFFFFFFFFull || workspace_bytes < gtr_xs_sorted_workspace_bytes(n) ||
+        (uint64_t)tables->n_union >= (1ull << 28) || (cfg->flags & GTR_F_HISTORY))
+        return GTR_EINVAL;
+    if (!valid_cfg(cfg)) return GTR_EINVAL;
+    cudaStream_t s = static_cast<cudaStream_t>(stream);
+    uint32_t *key = static_cast<uint32_t *>(d_workspace);
+    uint32_t *mu = key + n, *perm = key + 2 * n, *smu = key + 3 * n, *hist = key + 4 * n;
+    xs::Params P = xs::make_params(tables, first, n, seed, d_out, verify, nullptr);
+    GTR_CUDA_TRY(cudaMemsetAsync(hist, 0, 4u * xs::kSortBins, s));
+    xs::k_sort_sample<<<grid_blocks(ctx, (int64_t)n, 256), 256, 0, s>>>(P, key, mu, hist);
+    xs::k_sort_scan_local<<<xs::kScanBlocks, 1024, 0, s>>>(hist, hist + xs::kSortBins);
+    xs::k_sort_scan_add<<<xs::kScanBlocks, 1024, 0, s>>>(hist, hist + xs::kSortBins);
+    xs::k_sort_scatter<<<grid_blocks(ctx, (int64_t)n, 256), 256, 0, s>>>(n, key, mu, hist, perm, smu);
+    GTR_CUDA_TRY(cudaGetLastError());
+    P.s_perm = perm;
+    P.s_mu = smu;
+    xs::LaunchArgs a{ctx, cfg, P, s, nullptr};
+    return xs::launch(a);
 }

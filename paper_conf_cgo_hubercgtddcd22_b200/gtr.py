@@ -21,7 +21,7 @@ _lib = C.CDLL(LIB_PATH)
 GTR_OK, GTR_EINVAL, GTR_ECUDA, GTR_ENOMEM, GTR_EHEAP, GTR_EDEVICE, GTR_EUNSUPPORTED = 0, -1, -2, -3, -4, -5, -6
 GENERIC, GENERIC_CASCADE, CSM, SPMD, NATIVE = 0, 1, 2, 3, 4
 PL_RUNTIME, PL_GLOBAL, PL_SHARED_STATIC, PL_STACK, PL_COALESCED = 0, 1, 2, 3, 4
-F_BCAST_1BAR, F_SEPARATE_GUARDS, F_PLAIN = 1, 2, 4
+F_BCAST_1BAR, F_SEPARATE_GUARDS, F_PLAIN, F_HISTORY = 1, 2, 4, 8
 K_XS, K_SU3, K_RS, K_FORKJOIN, K_SEMANTICS, K_BARRIER_FLOOR = 0, 1, 2, 3, 4, 5
 MODE_NAMES = {GENERIC: "generic", GENERIC_CASCADE: "cascade", CSM: "csm", SPMD: "spmd", NATIVE: "native"}
 PL_NAMES = {PL_RUNTIME: "runtime", PL_GLOBAL: "global", PL_SHARED_STATIC: "shared_static", PL_STACK: "stack",
@@ -102,6 +102,9 @@ _proto = {
     "gtr_xs_build_hash_grid": (_i, [_vp, _vp, _i64, _i64, C.c_int32, _vp, _vp]),
     "gtr_xs_lookup": (_i, [_vp, _P(gtr_launch_cfg), _P(gtr_xs_tables), _u64, _u64, _u64, _vp,
                            _P(gtr_xs_verify), _vp]),
+    "gtr_xs_sorted_workspace_bytes": (_u64, [_u64]),
+    "gtr_xs_lookup_sorted": (_i, [_vp, _P(gtr_launch_cfg), _P(gtr_xs_tables), _u64, _u64, _u64, _vp,
+                                  _P(gtr_xs_verify), _vp, _u64, _vp]),
     "gtr_xs_lookup_host": (_i, [_vp, _P(gtr_launch_cfg), _P(gtr_xs_tables), _P(gtr_xs_request), _vp, _vp]),
     "gtr_l2_persist": (_i, [_vp, _vp, _u64, _u64, C.c_float, _vp]),
     "gtr_su3_mat_nn": (_i, [_vp, _P(gtr_launch_cfg), _vp, _vp, _vp, _i64, C.c_int32, _vp]),
@@ -220,6 +223,19 @@ def gtr_xs_lookup(ctx, launch_cfg, tables, first, n, seed, d_out, verify=None, s
     return _check("gtr_xs_lookup", _lib.gtr_xs_lookup(ctx, C.byref(launch_cfg), C.byref(tables), first, n, seed,
                                                       _ptr(d_out), C.byref(verify) if verify else None,
                                                       _stream(stream)))
+
+
+def gtr_xs_sorted_workspace_bytes(n):
+    return _lib.gtr_xs_sorted_workspace_bytes(n)
+
+
+def gtr_xs_lookup_sorted(ctx, launch_cfg, tables, first, n, seed, d_out, d_workspace, verify=None, stream=None):
+    """d_workspace: a device tensor of at least gtr_xs_sorted_workspace_bytes(n) bytes."""
+    nbytes = d_workspace.numel() * d_workspace.element_size()
+    return _check("gtr_xs_lookup_sorted",
+                  _lib.gtr_xs_lookup_sorted(ctx, C.byref(launch_cfg), C.byref(tables), first, n, seed, _ptr(d_out),
+                                            C.byref(verify) if verify else None, _ptr(d_workspace), nbytes,
+                                            _stream(stream)))
 
 
 def gtr_xs_lookup_host(ctx, launch_cfg, tables, h_req, h_out, stream=None):

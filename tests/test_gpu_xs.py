@@ -170,6 +170,61 @@ def test_grid_types_native(G, ctx, dev_grid, small):
     assert np.array_equal(v["macro"].view(np.uint64), o_v["macro"].view(np.uint64))
 
 
+# ---------------------------------------------------------------- SURVEY NEXT f2
+@pytest.mark.parametrize("variant", all_variants((128, 256)) + [(4, 3, 1, 128), (4, 3, 1, 256)], ids=vid)
+def test_history_mode_bit_exact(G, ctx, dev_small, small, variant):
+    """XSBench's history-based mode: a thread = a particle of 34 consecutive
+    lookups; same sampling, so the same results."""
+    t, P, o_out, o_v, n = small
+    m, p, f, nt = variant
+    out, v = _run(G, ctx, dev_small, G.cfg(m, p, f, nt, flags=G.F_HISTORY), 0, n)
+    _assert_same(out, v, o_out, o_v)
+
+
+def _run_sorted(G, ctx, dev, cfg, first, n):
+    out = torch.zeros(18, dtype=torch.uint64, device="cuda")
+    v, bufs = dev.verify_buffers(n)
+    ws = torch.empty(G.gtr_xs_sorted_workspace_bytes(n), dtype=torch.uint8, device="cuda")
+    G.gtr_xs_lookup_sorted(ctx, cfg, dev.tables, first, n, X.SEED_L, out, ws, v)
+    G.gtr_ctx_check(ctx)
+    return out.cpu().numpy(), {k: b.cpu().numpy() for k, b in bufs.items()}
+
+
+@pytest.mark.parametrize("variant", all_variants((256,)) + [(4, 3, 1, 256)], ids=vid)
+def test_sorted_mode_bit_exact(G, ctx, dev_small, small, variant):
+    """Lookups counting-sorted by (material, energy) before the lookup pass:
+    per-lookup records (indexed by lookup) and tallies identical."""
+    t, P, o_out, o_v, n = small
+    m, p, f, nt = variant
+    out, v = _run_sorted(G, ctx, dev_small, G.cfg(m, p, f, nt), 0, n)
+    _assert_same(out, v, o_out, o_v)
+
+
+@pytest.mark.parametrize("first,n", [(0, 1), (31337, 4097), (3, 70001)])
+def test_sorted_mode_ragged(G, ctx, dev_small, small, first, n):
+    t, P, *_ = small
+    o_out, o_v = P.run(first, n, X.SEED_L, 4, verify=True)
+    for mode in (G.SPMD, G.GENERIC, G.NATIVE):
+        for flags in (0, G.F_PLAIN):                 # staged nuclide loops / whole lookups per thread
+            out, v = _run_sorted(G, ctx, dev_small, G.cfg(mode, G.PL_STACK, 1, 128, flags=flags), first, n)
+            _assert_same(out, v, o_out, o_v)
+
+
+def test_sorted_mode_grid_types(G, ctx, dev_grid, small):
+    gt, dev = dev_grid
+    t, P, o_out, o_v, n = small
+    out, v = _run_sorted(G, ctx, dev, G.cfg(G.SPMD, G.PL_STACK, 1, 256), 0, n)
+    assert np.array_equal(out, o_out)
+    assert np.array_equal(v["macro"].view(np.uint64), o_v["macro"].view(np.uint64))
+
+
+def test_sorted_mode_rejects_small_workspace(G, ctx, dev_small):
+    out = torch.zeros(18, dtype=torch.uint64, device="cuda")
+    ws = torch.empty(1024, dtype=torch.uint8, device="cuda")
+    with pytest.raises(G.GtrError):
+        G.gtr_xs_lookup_sorted(ctx, G.cfg(), dev_small.tables, 0, 1000, X.SEED_L, out, ws)
+
+
 def test_variant_resources(G):
     info = G.gtr_query_variant(G.K_XS, G.cfg(G.SPMD, G.PL_STACK, 1, 256))
     assert info["block_threads"] == 256 and info["regs"] > 0 and info["num_teams"] > 0

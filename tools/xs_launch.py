@@ -25,6 +25,14 @@ VARIANTS = {
     "csm": G.cfg(G.CSM, G.PL_STACK, 1, 256),
     "csm128": G.cfg(G.CSM, G.PL_STACK, 1, 128),
     "generic": G.cfg(G.GENERIC, G.PL_STACK, 1, 256),
+    "spmd_history": G.cfg(G.SPMD, G.PL_STACK, 1, 256, flags=G.F_HISTORY),
+    "native_history": G.cfg(G.NATIVE, G.PL_STACK, 1, 256, flags=G.F_HISTORY),
+    "spmd_sorted": G.cfg(G.SPMD, G.PL_STACK, 1, 256),
+    "spmd128_sorted": G.cfg(G.SPMD, G.PL_STACK, 1, 128),
+    "spmd_plain_sorted": G.cfg(G.SPMD, G.PL_STACK, 1, 256, flags=G.F_PLAIN),
+    "native_sorted": G.cfg(G.NATIVE, G.PL_STACK, 1, 256),
+    "csm_sorted": G.cfg(G.CSM, G.PL_STACK, 1, 256),
+    "generic_sorted": G.cfg(G.GENERIC, G.PL_STACK, 1, 256),
 }
 
 ap = argparse.ArgumentParser()
@@ -42,16 +50,23 @@ out = torch.zeros(18, dtype=torch.uint64, device="cuda")
 if a.persist > 0:
     G.gtr_l2_persist(ctx, xs.grid, xs.grid.numel() * 8, a.persist_mb << 20, a.persist)
     print("persist window", a.persist, a.persist_mb, "MB")
+ws = None
 for v in a.variants:
     c = VARIANTS[v]
     out.zero_()
-    G.gtr_xs_lookup(ctx, c, xs.tables, 0, a.n, X.SEED_L, out)
+    if v.endswith("_sorted"):
+        if ws is None:
+            ws = torch.empty(G.gtr_xs_sorted_workspace_bytes(a.n), dtype=torch.uint8, device="cuda")
+        run = lambda: G.gtr_xs_lookup_sorted(ctx, c, xs.tables, 0, a.n, X.SEED_L, out, ws)  # noqa: E731
+    else:
+        run = lambda: G.gtr_xs_lookup(ctx, c, xs.tables, 0, a.n, X.SEED_L, out)  # noqa: E731
+    run()
     if a.time:
         e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         e0.record()
         for _ in range(a.reps):
             out.zero_()
-            G.gtr_xs_lookup(ctx, c, xs.tables, 0, a.n, X.SEED_L, out)
+            run()
         e1.record()
         torch.cuda.synchronize()
         ms = e0.elapsed_time(e1) / a.reps
