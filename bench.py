@@ -444,10 +444,16 @@ def su3_sweep(G, torch, ctx, stream):
                     ("generic", G.cfg(G.GENERIC, G.PL_STACK, 1, 64)),
                     ("generic_runtime_globalized", G.cfg(G.GENERIC, G.PL_RUNTIME, 0, 64)),
                     ("generic_llvm12_coalesced", G.cfg(G.GENERIC, G.PL_COALESCED, 0, 64)),
-                    ("csm_shared_fold", G.cfg(G.CSM, G.PL_SHARED_STATIC, 1, 64))]:
+                    ("csm_shared_fold", G.cfg(G.CSM, G.PL_SHARED_STATIC, 1, 64)),
+                    # GTR_F_TMA: sequential code streams 16-site tiles with bulk async copies
+                    ("native_tma", G.cfg(G.NATIVE, G.PL_STACK, 1, 256, flags=G.F_TMA)),
+                    ("spmd_tma", G.cfg(G.SPMD, G.PL_STACK, 1, 64, flags=G.F_TMA)),
+                    ("csm_tma", G.cfg(G.CSM, G.PL_STACK, 1, 128, flags=G.F_TMA)),
+                    ("generic_tma", G.cfg(G.GENERIC, G.PL_STACK, 1, 128, flags=G.F_TMA))]:
         ms = _time(torch, stream, lambda: G.gtr_su3_mat_nn(ctx, c, dA, dB, dC, sites, 1, stream), 3)
         ok = bool(torch.all(dC.view(-1, 2)[:, 0] == 1.0).item()) and bool(torch.all(dC.view(-1, 2)[:, 1] == 0.0).item())
         res[name] = {"ms_per_iter": ms, "gb_s": sites * 1152 / (ms * 1e-3) / 1e9,
+                     "hbm_frac": sites * 1152 / (ms * 1e-3) / 1e9 / peaks()[0],
                      "regs": G.gtr_query_variant(G.K_SU3, c)["regs"], "closed_form_ok": ok}
     G.gtr_ctx_check(ctx, stream)
     del dA, dC
@@ -529,7 +535,9 @@ def sharded_apps(G, torch, ctx, rank, ws, dist, stream, dev):
     dA, dB = su3_device(A, B, device=dev)
     del A
     dC = torch.empty_like(dA)
-    for name, cc in (("native", G.cfg(G.NATIVE, G.PL_STACK, 1, 256)), ("spmd", G.cfg(G.SPMD, G.PL_STACK, 1, 64))):
+    for name, cc in (("native", G.cfg(G.NATIVE, G.PL_STACK, 1, 256)), ("spmd", G.cfg(G.SPMD, G.PL_STACK, 1, 64)),
+                     ("native_tma", G.cfg(G.NATIVE, G.PL_STACK, 1, 256, flags=G.F_TMA)),
+                     ("spmd_tma", G.cfg(G.SPMD, G.PL_STACK, 1, 64, flags=G.F_TMA))):
         ms = _time(torch, stream, lambda: G.gtr_su3_mat_nn(ctx, cc, dA, dB, dC, m, 1, stream), 3)
         ok = bool(torch.all(dC.view(-1, 2)[:, 0] == 1.0).item()) and bool(torch.all(dC.view(-1, 2)[:, 1] == 0.0).item())
         t = torch.tensor([ms, 0.0 if ok else 1.0], dtype=torch.float64, device=dev)

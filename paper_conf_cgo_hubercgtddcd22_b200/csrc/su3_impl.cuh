@@ -10,8 +10,16 @@
 // with 4 complex temporaries (accumulator, a, b, product) whose addresses are
 // taken by the complex operators -> globalized (AMB-7).  fp64 (AMB-8); every
 // product rounded before the add/sub (this TU: -fmad=false).
+//
+// GTR_F_TMA (B200-native form of the same program): `teams distribute` over
+// tiles of 16 sites; the team's sequential code -- main thread (generic) or a
+// guard (SPMD) -- issues bulk asynchronous copies (the TMA engine): the next
+// tile's A into a second shared buffer while the current tile's parallel
+// region runs, and the finished C tile back to HBM.  Regions read A and write C
+// in shared memory; HBM traffic is whole-tile streaming.  Same arithmetic.
 #pragma once
 #include "gtr_internal.h"
+#include "tma.cuh"
 
 namespace gtr {
 namespace su3 {
@@ -21,6 +29,7 @@ struct Params {
     const double2 *B;   // [4][3][3]
     double2 *C;
     int64_t sites;
+    int32_t tma;        // GTR_F_TMA: tile-streamed form
 };
 static __shared__ Params g_p;
 
@@ -41,8 +50,10 @@ __device__ __forceinline__ void cadd_to(double *acc, const double *p) {
     acc[1] = acc[1] + p[1];
 }
 
-// one output element e = (j, k, l) of site s
-template <class K> __device__ __forceinline__ void element(const Params &P, int64_t s, int e) {
+// one output element e = (j, k, l) of a site whose 36 A values start at
+// `As` (global or shared) -> *out
+template <class K, bool GLOBAL_A>
+__device__ __forceinline__ void element_at(const double2 *As, const double2 *B, int e, double2 *out) {
     const int j = e / 9, k = (e / 3) % 3, l = e % 3;
     Local<K, double, 2, TagCC> cc;
     Local<K, double, 2, TagA> a;
@@ -52,14 +63,86 @@ template <class K> __device__ __forceinline__ void element(const Params &P, int6
     cc[1] = 0.0;
 #pragma unroll
     for (int m = 0; m < 3; m++) {
-        const double2 av = __ldg(P.A + ((s * 4 + j) * 3 + k) * 3 + m);
-        const double2 bv = __ldg(P.B + (j * 3 + m) * 3 + l);
+        const double2 av = GLOBAL_A ? __ldg(As + (j * 3 + k) * 3 + m) : As[(j * 3 + k) * 3 + m];
+        const double2 bv = __ldg(B + (j * 3 + m) * 3 + l);
         a[0] = av.x; a[1] = av.y;
         b[0] = bv.x; b[1] = bv.y;
         cmul(p.ptr(), a.ptr(), b.ptr());
         cadd_to(cc.ptr(), p.ptr());
     }
-    P.C[((s * 4 + j) * 3 + k) * 3 + l] = make_double2(cc[0], cc[1]);
+    *out = make_double2(cc[0], cc[1]);
+}
+// one output element e = (j, k, l) of site s
+template <class K> __device__ __forceinline__ void element(const Params &P, int64_t s, int e) {
+    element_at<K, true>(P.A + s * 36, P.B, e, P.C + s * 36 + e);
+}
+
+// ---- GTR_F_TMA: tile buffers in dynamic shared memory after the runtime's area
+constexpr int kTileSites = 16;
+constexpr uint32_t kSiteBytes = 36 * 16;
+struct TileBuf {
+    double2 a[2][kTileSites * 36];   // double-buffered A tiles (TMA destinations)
+    double2 c[kTileSites * 36];      // C tile (TMA store source)
+    uint64_t bar[2];                 // completion barriers of the A buffers
+};
+template <class K> __device__ __forceinline__ TileBuf &tile_buf() {
+    const uint32_t off = tstate_bytes<K>() + (uint32_t)K::BLOCK * g_ts.rp.sm_stride_words * 8u;
+    return *reinterpret_cast<TileBuf *>(g_dyn + ((off + 127u) & ~127u));
+}
+struct TileArgs {
+    int32_t ns;        // sites in this tile
+    int32_t buf;       // A buffer
+    uint32_t parity;   // phase parity of that buffer's barrier
+};
+struct TagTile {};
+template <class K> struct TileRegion {
+    static constexpr int ID = 2;
+    static __device__ void run(void *a) {
+        const TileArgs *t = static_cast<const TileArgs *>(a);
+        TileBuf &tb = tile_buf<K>();
+        tma::mbar_wait(&tb.bar[t->buf], t->parity);             // A tile landed
+        const double2 *At = tb.a[t->buf];
+        for_static<K>(0, (int64_t)t->ns * 36, [&](int64_t q) {
+            const int site = (int)(q / 36), e = (int)(q - site * 36);
+            element_at<K, false>(At + site * 36, g_p.B, e, &tb.c[q]);
+        });
+        tma::fence_async_shared();                               // C writes before the bulk store
+    }
+};
+// the team's sequential program of the tiled form
+template <class K> __device__ __forceinline__ void team_program_tma() {
+    TileBuf &tb = tile_buf<K>();
+    const int64_t ntiles = (g_p.sites + kTileSites - 1) / kTileSites;
+    const int64_t t0 = team_num<K>(), G = num_teams<K>();
+    auto tile_sites = [&](int64_t t) {
+        return (int32_t)((t + 1) * kTileSites <= g_p.sites ? kTileSites : g_p.sites - t * kTileSites);
+    };
+    guarded<K>([&] {
+        tma::mbar_init(&tb.bar[0]);
+        tma::mbar_init(&tb.bar[1]);
+        tma::fence_mbar_init();
+        if (t0 < ntiles)
+            tma::load_async(tb.a[0], g_p.A + t0 * kTileSites * 36, (uint32_t)tile_sites(t0) * kSiteBytes, &tb.bar[0]);
+    });
+    int i = 0;
+    for (int64_t t = t0; t < ntiles; t += G, i++) {
+        guarded<K>([&] {
+            const int64_t tn = t + G;                            // prefetch the next tile
+            if (tn < ntiles)
+                tma::load_async(tb.a[(i + 1) & 1], g_p.A + tn * kTileSites * 36,
+                                (uint32_t)tile_sites(tn) * kSiteBytes, &tb.bar[(i + 1) & 1]);
+            tma::store_wait_read();                              // C buffer free again
+        });
+        TeamLocal<K, TileArgs, TagTile> args;
+        args.set([&](TileArgs &x) {
+            x.ns = tile_sites(t);
+            x.buf = i & 1;
+            x.parity = (uint32_t)((i >> 1) & 1);
+        });
+        parallel<K, TileRegion<K>>(args.get());
+        guarded<K>([&] { tma::store_async(g_p.C + t * kTileSites * 36, tb.c, (uint32_t)tile_sites(t) * kSiteBytes); });
+    }
+    guarded<K>([&] { tma::store_wait_all(); });
 }
 
 struct Site {
@@ -79,10 +162,15 @@ template <class K> __global__ void __launch_bounds__(K::BLOCK) kernel_rt(Params 
     const Role role = team_init<K>(rp);
     if (role == Role::Exit) return;
     if (role == Role::Worker) {
-        worker_loop<K, SiteRegion<K>>();
+        worker_loop<K, SiteRegion<K>, TileRegion<K>>();
         return;
     }
     guarded<K>([&] { g_p = P; });
+    if (P.tma) {
+        team_program_tma<K>();
+        team_deinit<K>();
+        return;
+    }
     for (int64_t s = team_num<K>(); s < P.sites; s += num_teams<K>()) {   // teams distribute
         TeamLocal<K, Site, TagSite> site;
         site.set([&](Site &x) { x.s = s; });
@@ -104,7 +192,7 @@ template <class K> struct OpRt {
     static int run(LaunchArgs &a) {
         const void *fn = reinterpret_cast<const void *>(&kernel_rt<K>);
         Launch L;
-        int st = resolve<K>(a.ctx, a.cfg, fn, 80, &L);
+        int st = resolve<K>(a.ctx, a.cfg, fn, 80, &L, false, a.P.tma ? (uint32_t)sizeof(TileBuf) + 128u : 0u);
         if (st) return st;
         if (a.info) {
             int per_sm = 0;

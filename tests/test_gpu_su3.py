@@ -50,3 +50,36 @@ def test_su3_full_lattice_constant_closed_form(G, ctx):
     for mode in (G.SPMD, G.NATIVE):
         got = _run(G, ctx, G.cfg(mode, G.PL_STACK, 1, 128), A, B, iters=1)
         assert (got.real == 1.0).all() and (got.imag == 0.0).all()
+
+
+@pytest.mark.parametrize("variant", list(itertools.product(RUNTIME_MODES, PLACEMENTS, (0, 1), (64, 128))),
+                         ids=lambda v: "m%d-p%d-f%d-t%d" % v)
+def test_su3_tma_all_variants_bit_exact(G, ctx, lattice, variant):
+    """GTR_F_TMA: the sequential code streams 16-site tiles with bulk async
+    copies (ragged last tile: 1303 sites = 81 x 16 + 7); same bits."""
+    A, B, want = lattice
+    m, p, f, nt = variant
+    for teams in (0, 5):                     # one wave / few teams (many tiles per team)
+        got = _run(G, ctx, G.cfg(m, p, f, nt, num_teams=teams, flags=G.F_TMA), A, B)
+        assert np.array_equal(got.view(np.uint64), want.view(np.uint64)), teams
+
+
+@pytest.mark.parametrize("nt", (128, 256, 512))
+def test_su3_native_tma_bit_exact(G, ctx, lattice, nt):
+    A, B, want = lattice
+    for teams in (0, 3):
+        got = _run(G, ctx, G.cfg(G.NATIVE, G.PL_STACK, 1, nt, num_teams=teams, flags=G.F_TMA), A, B)
+        assert np.array_equal(got.view(np.uint64), want.view(np.uint64)), teams
+
+
+def test_su3_tma_tiny_and_full(G, ctx, orc):
+    for sites in (1, 15, 17):
+        A, B = S.make_lattice(sites, "random")
+        want = orc.su3_mat_nn(A, B)
+        for mode in (G.SPMD, G.GENERIC, G.NATIVE):
+            got = _run(G, ctx, G.cfg(mode, G.PL_STACK, 1, 128, flags=G.F_TMA), A, B)
+            assert np.array_equal(got.view(np.uint64), want.view(np.uint64)), (sites, mode)
+    A, B = S.make_lattice(32 ** 4, "constant")
+    for mode in (G.SPMD, G.NATIVE):
+        got = _run(G, ctx, G.cfg(mode, G.PL_STACK, 1, 128, flags=G.F_TMA), A, B, iters=1)
+        assert (got.real == 1.0).all() and (got.imag == 0.0).all()
