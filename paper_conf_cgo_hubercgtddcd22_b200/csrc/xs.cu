@@ -216,12 +216,12 @@ extern "C" int gtr_xs_build_hash_grid(gtr_ctx *ctx, const double *d_energies, in
 
 static bool tables_ok(const gtr_xs_tables *t) {
     if (!(t && t->grid && t->num_nucs && t->mats && t->concs && t->n_iso > 0 && t->n_gp >= 2 &&
-          t->max_num_nucs > 0 && t->n_iso * t->n_gp < (int64_t)UINT32_MAX))
+          t->max_num_nucs > 0 && t->n_iso * t->n_gp < ((int64_t)1 << 28)))   // u packs in 28 bits
         return false;
     switch (t->grid_type) {
     case GTR_XS_UNIONIZED: return t->egrid && t->index_grid && t->n_union >= 2;
     case GTR_XS_NUCLIDE: return t->energies != nullptr;
-    case GTR_XS_HASH: return t->energies && t->hash_index && t->hash_bins >= 1;
+    case GTR_XS_HASH: return t->energies && t->hash_index && t->hash_bins >= 1 && t->hash_bins < (1 << 28);
     default: return false;
     }
 }
