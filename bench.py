@@ -98,9 +98,12 @@ def dist_init():
     ws = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
-    if ws > 1:
+    if ws > 1 or os.environ.get("GTR_BENCH_DIST") == "1":   # GTR_BENCH_DIST: exercise the N>1 path on 1 GPU
         import torch.distributed as dist
         os.environ.setdefault("MASTER_ADDR", "127.0.0.1")
+        os.environ.setdefault("MASTER_PORT", "29517")
+        os.environ.setdefault("RANK", "0")
+        os.environ.setdefault("WORLD_SIZE", str(ws))
         torch.cuda.set_device(local)
         dist.init_process_group("nccl", device_id=torch.device("cuda", local))
     else:
@@ -161,8 +164,9 @@ def run_gtr(a):
 
     ws, rank, local = dist_init()
     dist = None
-    if ws > 1:
-        import torch.distributed as dist
+    import torch.distributed as _d
+    if _d.is_initialized():
+        dist = _d
     dev = torch.device("cuda", local)
     stream = torch.cuda.current_stream()
     pool = torch.zeros(64 << 20, dtype=torch.uint8, device=dev)
@@ -180,7 +184,26 @@ def run_gtr(a):
     out = torch.zeros(18, dtype=torch.uint64, device=dev)
     num_nucs = tables["num_nucs"].astype(np.int64)
 
+    # N > 1: the 18-u64 combine is fused into the lookup kernel's epilogue
+    # (teams add into every rank's buffer over NVLink peer memory, then one
+    # device barrier; dist.PeerCombine); NCCL all_reduce only if the
+    # symmetric-memory rendezvous is unavailable on the box
+    pc, combine = None, None
+    if dist is not None:
+        from paper_conf_cgo_hubercgtddcd22_b200.dist import PeerCombine
+        try:
+            pc = PeerCombine(dev)
+            combine = "fused: team epilogue adds into every rank's buffer over NVLink peer memory + device barrier"
+        except Exception as e:  # noqa: BLE001 -- collective implementation choice, reported in the line
+            pc = None
+            combine = f"NCCL all_reduce (peer-memory rendezvous unavailable: {type(e).__name__})"
+
     def step():
+        nonlocal out
+        if pc is not None:
+            G.gtr_xs_lookup_peers(ctx, head, xs.tables, first, n, seed, pc.ptrs(), stream)
+            out = pc.finish()
+            return
         out.zero_()
         G.gtr_xs_lookup(ctx, head, xs.tables, first, n, seed, out, None, stream)
         if dist is not None:
@@ -200,6 +223,13 @@ def run_gtr(a):
         torch.cuda.synchronize()
         e0.record(stream)
         for s in range(a.steps):
+            if pc is not None:
+                ptrs = pc.ptrs()
+                kev[s][0].record(stream)
+                G.gtr_xs_lookup_peers(ctx, head, xs.tables, first, n, seed, ptrs, stream)
+                kev[s][1].record(stream)
+                out = pc.finish()
+                continue
             out.zero_()
             kev[s][0].record(stream)
             G.gtr_xs_lookup(ctx, head, xs.tables, first, n, seed, out, None, stream)
@@ -272,8 +302,8 @@ def run_gtr(a):
             "warmup": a.warmup, "ms_per_step": ms, "higher_is_better": True, "scaling": "weak",
             "vs_baseline": None, "dtype": "f64", "data": "synthetic",
             "config": {"workload": WORKLOAD, "variant": "SPMD + heap-to-stack + folding, thread_limit 256",
-                       "lookups_per_gpu": n, "parallelism": f"lookups sharded over {ws} GPU(s), NCCL all-reduce "
-                                                             "of hash+tallies" if ws > 1 else "1 GPU",
+                       "lookups_per_gpu": n, "parallelism": f"lookups sharded over {ws} GPU(s); combine of "
+                                                             f"hash+tallies: {combine}" if dist is not None else "1 GPU",
                        "l2": "no flush: inputs 5.9 GB per GPU >> 126 MB L2 (index grid 5.7 GB)",
                        "table_setup_s": round(t_setup, 2)},
             "hash": int(res[0]), "hash_mod_999983": int(res[0] % 999983),

@@ -31,7 +31,7 @@ template <int NT> __global__ void __launch_bounds__(NT) kernel_native(Params P) 
             lookup<KN>(P, P.first + k, tally);
     }
     __syncthreads();
-    flush(tally, P.out, threadIdx.x, NT);
+    flush_out(P, tally, threadIdx.x, NT);
 }
 
 // ---------------------------------------------------------------- builders
@@ -353,5 +353,19 @@ extern "C" int gtr_xs_lookup_sorted(gtr_ctx *ctx, const gtr_launch_cfg *cfg, con
     P.s_perm = perm;
     P.s_mu = smu;
     xs::LaunchArgs a{ctx, cfg, P, s, nullptr};
+    return xs::launch(a);
+}
+
+extern "C" int gtr_xs_lookup_peers(gtr_ctx *ctx, const gtr_launch_cfg *cfg, const gtr_xs_tables *tables,
+                                   uint64_t first, uint64_t n, uint64_t seed, uint64_t *const *h_peer_outs,
+                                   int32_t n_peers, void *stream) {
+    if (!ctx || !cfg || !tables_ok(tables) || !h_peer_outs || n_peers < 1 || n_peers > 8) return GTR_EINVAL;
+    for (int p = 0; p < n_peers; p++)
+        if (!h_peer_outs[p]) return GTR_EINVAL;
+    if (n == 0) return GTR_OK;
+    xs::Params P = xs::make_params(tables, first, n, seed, h_peer_outs[0], nullptr, nullptr);
+    P.n_peers = n_peers;
+    for (int p = 0; p < n_peers; p++) P.peer_out[p] = reinterpret_cast<unsigned long long *>(h_peer_outs[p]);
+    xs::LaunchArgs a{ctx, cfg, P, static_cast<cudaStream_t>(stream), nullptr};
     return xs::launch(a);
 }

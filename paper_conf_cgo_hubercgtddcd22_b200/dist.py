@@ -59,3 +59,39 @@ def gather_shards(local, group=None):
     parts = [torch.empty_like(local) for _ in range(dist.get_world_size(group))]
     dist.all_gather(parts, local.contiguous(), group=group)
     return torch.cat(parts, 0)
+
+
+class PeerCombine:
+    """The 18-u64 all-reduce of the sharded XS step fused into the lookup
+    kernel (gtr_xs_lookup_peers): every rank's teams add their tallies
+    straight into every rank's result buffer over NVLink peer memory
+    (system-scope atomics), then one device-side barrier.  The buffers are a
+    torch symmetric-memory allocation (peer mappings of each rank's slot);
+    two slots alternate so the next step's slot is zeroed before the barrier
+    that precedes anyone's next kernel.  Integer sums: bit-identical to the
+    NCCL all-reduce for any world size.
+
+    Per step:  ptrs() -> launch gtr_xs_lookup_peers(..., ptrs) -> finish()
+    (zero the other local slot, barrier on the current stream) -> the local
+    slot holds the combined result."""
+
+    def __init__(self, device, group=None):
+        import torch.distributed as dist
+        import torch.distributed._symmetric_memory as symm_mem
+        g = group or dist.group.WORLD
+        self.buf = symm_mem.empty(36, dtype=torch.int64, device=device).view(2, 18)
+        self.handle = symm_mem.rendezvous(self.buf, g.group_name)
+        self.buf.zero_()
+        self.handle.barrier()
+        self.step = 0
+
+    def ptrs(self):
+        off = (self.step % 2) * 18 * 8
+        return [int(p) + off for p in self.handle.buffer_ptrs]
+
+    def finish(self):
+        b = self.step % 2
+        self.buf[1 - b].zero_()
+        self.handle.barrier()
+        self.step += 1
+        return self.buf[b].view(torch.uint64)

@@ -105,6 +105,8 @@ _proto = {
     "gtr_xs_sorted_workspace_bytes": (_u64, [_u64]),
     "gtr_xs_lookup_sorted": (_i, [_vp, _P(gtr_launch_cfg), _P(gtr_xs_tables), _u64, _u64, _u64, _vp,
                                   _P(gtr_xs_verify), _vp, _u64, _vp]),
+    "gtr_xs_lookup_peers": (_i, [_vp, _P(gtr_launch_cfg), _P(gtr_xs_tables), _u64, _u64, _u64, _P(_u64), C.c_int32,
+                                 _vp]),
     "gtr_xs_lookup_host": (_i, [_vp, _P(gtr_launch_cfg), _P(gtr_xs_tables), _P(gtr_xs_request), _vp, _vp]),
     "gtr_l2_persist": (_i, [_vp, _vp, _u64, _u64, C.c_float, _vp]),
     "gtr_su3_mat_nn": (_i, [_vp, _P(gtr_launch_cfg), _vp, _vp, _vp, _i64, C.c_int32, _vp]),
@@ -236,6 +238,14 @@ def gtr_xs_lookup_sorted(ctx, launch_cfg, tables, first, n, seed, d_out, d_works
                   _lib.gtr_xs_lookup_sorted(ctx, C.byref(launch_cfg), C.byref(tables), first, n, seed, _ptr(d_out),
                                             C.byref(verify) if verify else None, _ptr(d_workspace), nbytes,
                                             _stream(stream)))
+
+
+def gtr_xs_lookup_peers(ctx, launch_cfg, tables, first, n, seed, peer_ptrs, stream=None):
+    """peer_ptrs: device addresses (ints) of every rank's 18-u64 result buffer."""
+    arr = (_u64 * len(peer_ptrs))(*peer_ptrs)
+    return _check("gtr_xs_lookup_peers",
+                  _lib.gtr_xs_lookup_peers(ctx, C.byref(launch_cfg), C.byref(tables), first, n, seed, arr,
+                                           len(peer_ptrs), _stream(stream)))
 
 
 def gtr_xs_lookup_host(ctx, launch_cfg, tables, h_req, h_out, stream=None):

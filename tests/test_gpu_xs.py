@@ -225,6 +225,51 @@ def test_sorted_mode_rejects_small_workspace(G, ctx, dev_small):
         G.gtr_xs_lookup_sorted(ctx, G.cfg(), dev_small.tables, 0, 1000, X.SEED_L, out, ws)
 
 
+# ---------------------------------------------------------------- fused combine (8(e), f1)
+@pytest.mark.parametrize("mode", (0, 2, 3, 4))
+def test_peer_combine_epilogue(G, ctx, dev_small, small, mode):
+    """gtr_xs_lookup_peers adds every team's tallies into each listed buffer:
+    listing the same buffer k times must give exactly k x the oracle (u64
+    wrap-around), listing distinct buffers gives each the oracle's result."""
+    t, P, o_out, o_v, n = small
+    c = G.cfg(mode, G.PL_STACK, 1, 128)
+    buf = torch.zeros(18, dtype=torch.uint64, device="cuda")
+    G.gtr_xs_lookup_peers(ctx, c, dev_small.tables, 0, n, X.SEED_L, [buf.data_ptr()] * 3)
+    G.gtr_ctx_check(ctx)
+    assert np.array_equal(buf.cpu().numpy(), (o_out * np.uint64(3)).astype(np.uint64))
+    bufs = torch.zeros((8, 18), dtype=torch.uint64, device="cuda")
+    G.gtr_xs_lookup_peers(ctx, c, dev_small.tables, 0, n, X.SEED_L, [bufs[k].data_ptr() for k in range(8)])
+    G.gtr_ctx_check(ctx)
+    for k in range(8):
+        assert np.array_equal(bufs[k].cpu().numpy(), o_out), k
+
+
+def test_peer_combine_symmetric_memory_single_rank(G, ctx, dev_small, small):
+    """The PeerCombine plumbing (torch symmetric memory, device barrier) at
+    world size 1: three steps through the alternating slots."""
+    import os
+    import socket
+    import torch.distributed as dist
+    from paper_conf_cgo_hubercgtddcd22_b200.dist import PeerCombine
+    t, P, o_out, o_v, n = small
+    if not dist.is_initialized():
+        s = socket.socket()
+        s.bind(("127.0.0.1", 0))
+        port = s.getsockname()[1]
+        s.close()
+        os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port), RANK="0", WORLD_SIZE="1")
+        dist.init_process_group("nccl", device_id=torch.device("cuda", 0))
+    try:
+        pc = PeerCombine(torch.device("cuda", 0))
+        for _ in range(3):
+            G.gtr_xs_lookup_peers(ctx, G.cfg(G.SPMD, G.PL_STACK, 1, 256), dev_small.tables, 0, n, X.SEED_L,
+                                  pc.ptrs())
+            res = pc.finish()
+            assert np.array_equal(res.cpu().numpy(), o_out)
+    finally:
+        dist.destroy_process_group()
+
+
 def test_variant_resources(G):
     info = G.gtr_query_variant(G.K_XS, G.cfg(G.SPMD, G.PL_STACK, 1, 256))
     assert info["block_threads"] == 256 and info["regs"] > 0 and info["num_teams"] > 0
