@@ -172,3 +172,61 @@ def test_rs_work_counts_brute_force(orc, rs_small):
     # visits also equal sum over the material tallies of num_nucs
     out, _, _ = P.run(first, n, X.SEED_L)
     assert vis == int((out[1:13].astype(np.int64) * t["num_nucs"].astype(np.int64)).sum())
+
+
+# ---------------------------------------------------------------- sigT factors
+def _textbook_phi(l, rho):
+    """Hard-sphere phase shift phi_l = -delta_l, tan(delta_l) = j_l(rho) / y_l(rho)
+    (spherical Bessel functions; scipy), determined mod pi -- which the doubled
+    angle of the sigT factor exp(-2 i phi) does not see."""
+    from scipy.special import spherical_jn, spherical_yn
+    return -np.arctan(spherical_jn(l, rho) / spherical_yn(l, rho))
+
+
+@pytest.mark.parametrize("L", [0, 1, 2, 3])
+def test_sigT_factors_vs_spherical_bessel(orc, rs_small, L):
+    """Pins the oracle's sigT factors through whole
+    lookups: every window holds one pole of angular momentum L, background and
+    RA/RF are zero, so macro_T / sum(conc) = Re(RT * W(Z) * f_L(rho)).  Two runs
+    (RT = 1, RT = i) give W * f_L; dividing by the oracle's W (pinned against
+    wofz above) leaves f_L = exp(-2 i phi_L(rho)), rho = K0RS * sqrt(E).
+    l = 0, 2, 3 must equal the textbook hard-sphere phase shifts; l = 1 is
+    RSBench's `phi -= -atan(phi)`, i.e. rho + atan(rho) = 2 rho - phi_1 (the
+    textbook's correction with its sign flipped) -- pinned as such."""
+    K = 3.7                                  # rho up to ~3.7: crosses 3 - rho^2 = 0
+    EA = complex(0.41, -0.23)
+    got = {}
+    for name, RT in (("re", (1.0, 0.0)), ("im", (0.0, 1.0))):
+        t = {k: (v.copy() if isinstance(v, np.ndarray) else v) for k, v in rs_small.items()}
+        for f in ("T", "A", "F"):
+            t["windows"][f] = 0.0
+        t["windows"]["start"] = 0
+        t["windows"]["end"] = 1
+        p = t["poles"]
+        p["EA"][:, 0] = (EA.real, EA.imag)
+        p["RT"][:, 0] = RT
+        p["RA"][:, 0] = 0.0
+        p["RF"][:, 0] = 0.0
+        p["l_value"][:, 0] = L
+        t["k0rs"][:, L] = K
+        out, v, _ = orc.RsProblem(t).run(0, 300, X.SEED_L, 1, verify=True)
+        got[name] = v
+    n_checked = 0
+    for i, E in enumerate(energies(X.SEED_L, 300)):
+        mat = int(got["re"]["mat"][i])
+        csum = float(rs_small["concs"][mat, :int(rs_small["num_nucs"][mat])].sum())
+        a = got["re"]["macro"][i][0] / csum            # Re(W f)
+        b = got["im"]["macro"][i][0] / csum            # Re(i W f) = -Im(W f)
+        assert got["re"]["macro"][i][1] == 0.0 and got["re"]["macro"][i][2] == 0.0
+        Wf = complex(a, -b)
+        W = orc.fast_nuclear_W((E - EA) * 0.5)
+        f = Wf / W
+        rho = K * np.sqrt(E)
+        phi = _textbook_phi(L, rho)
+        if L == 1:
+            phi = 2.0 * rho - phi
+        want = np.exp(-2j * phi)
+        assert abs(f - want) <= 1e-11, (L, E, f, want)
+        assert abs(abs(f) - 1.0) <= 1e-11
+        n_checked += 1
+    assert n_checked == 300
