@@ -6,7 +6,9 @@ x 11,303 gridpoints, 17M lookups per GPU (weak scaling), synthetic seeded
 tables (gtr_inputs).  One step = one batch of 17M lookups through libgtr's
 headline variant (SPMD-ized + heap-to-stack + folding, thread_limit 256 --
 the paper's optimized form of XSBench's `target teams distribute parallel
-for`) plus, for N > 1, the NCCL all-reduce of the 18 u64 hash/tallies.
+for`) plus, for N > 1, the combine of the 18 u64 hash/tallies: fused into
+the kernel's epilogue over peer memory (dist.PeerCombine), checked once
+against an NCCL all-reduce after warm-up (NCCL is used if they differ).
 
     python bench.py [--gpus N] [--steps K] [--warmup W] [--impl gtr|reference]
     torchrun --nproc-per-node N bench.py --gpus N ...
@@ -212,6 +214,20 @@ def run_gtr(a):
     for _ in range(a.warmup):
         step()
     G.gtr_ctx_check(ctx, stream)
+    if pc is not None:
+        # one-time check of the fused combine against the NCCL all-reduce of
+        # this rank's own result (every box gpurun offers has one GPU, so the
+        # peer path is first exercised here); all ranks switch together
+        fused = out.clone()
+        loc = torch.zeros(18, dtype=torch.uint64, device=dev)
+        G.gtr_xs_lookup(ctx, head, xs.tables, first, n, seed, loc, None, stream)
+        combine_results(loc)
+        ok = torch.tensor([1 if torch.equal(fused.view(torch.int64), loc.view(torch.int64)) else 0], dtype=torch.int64, device=dev)
+        dist.all_reduce(ok, op=dist.ReduceOp.MIN)
+        if int(ok[0]) != 1:
+            pc = None
+            combine = "NCCL all_reduce (fused peer-memory combine failed its check against NCCL)"
+            step()
 
     # timed region: K steps, barrier + sync on both sides, CUDA events on the
     # launching stream; per-launch kernel events for the roofline

@@ -304,7 +304,13 @@ template <class K> struct BucketRegion {
 
 // 4 teams of 128 per SM: caps registers at 128 (measured +2% over the
 // unconstrained 146-register build, which fits 3)
-template <class K> __global__ void __launch_bounds__(K::BLOCK, K::NT == 128 ? 4 : 1) kernel_rt(Params P, RtParams rp) {
+#ifndef GTR_RS_MINB
+#define GTR_RS_MINB 4
+#endif
+#ifndef GTR_RS_MINB_GEN            // generic modes (thread_limit + 32 threads per team)
+#define GTR_RS_MINB_GEN 4
+#endif
+template <class K> __global__ void __launch_bounds__(K::BLOCK, K::NT == 128 ? (K::BLOCK > K::NT ? GTR_RS_MINB_GEN : GTR_RS_MINB) : 1) kernel_rt(Params P, RtParams rp) {
     const Role role = team_init<K>(rp);
     if (role == Role::Exit) return;
     if (role == Role::Worker) {
