@@ -214,10 +214,34 @@ extern "C" int gtr_xs_build_hash_grid(gtr_ctx *ctx, const double *d_energies, in
     return GTR_OK;
 }
 
+namespace gtr {
+namespace xs {
+// B[b] = #{m : egrid[m] < b / 2^L}, b in [0, 2^L] (b / 2^L exact in fp64)
+__global__ void k_union_bins(const double *__restrict__ egrid, int64_t n, int32_t log2b, uint32_t *__restrict__ out) {
+    const int64_t nb = (1ll << log2b) + 1;
+    for (int64_t b = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; b < nb; b += (int64_t)gridDim.x * blockDim.x)
+        out[b] = (uint32_t)count_below(egrid, n, (double)b / (double)(1ll << log2b), false);
+}
+}  // namespace xs
+}  // namespace gtr
+
+extern "C" int gtr_xs_build_union_bins(gtr_ctx *ctx, const double *d_egrid, int64_t n_union, int32_t log2_bins,
+                                       uint32_t *d_bins_out, void *stream) {
+    if (!ctx || !d_egrid || !d_bins_out || n_union < 2 || n_union >= ((int64_t)1 << 32) || log2_bins < 0 ||
+        log2_bins > 26)
+        return GTR_EINVAL;
+    const int64_t nb = ((int64_t)1 << log2_bins) + 1;
+    xs::k_union_bins<<<grid_blocks(ctx, nb, 256), 256, 0, static_cast<cudaStream_t>(stream)>>>(
+        d_egrid, n_union, log2_bins, d_bins_out);
+    GTR_CUDA_TRY(cudaGetLastError());
+    return GTR_OK;
+}
+
 static bool tables_ok(const gtr_xs_tables *t) {
     if (!(t && t->grid && t->num_nucs && t->mats && t->concs && t->n_iso > 0 && t->n_gp >= 2 &&
           t->max_num_nucs > 0 && t->n_iso * t->n_gp < ((int64_t)1 << 28)))   // u packs in 28 bits
         return false;
+    if (t->union_bins && (t->union_bins_log2 < 0 || t->union_bins_log2 > 26)) return false;
     switch (t->grid_type) {
     case GTR_XS_UNIONIZED: return t->egrid && t->index_grid && t->n_union >= 2;
     case GTR_XS_NUCLIDE: return t->energies != nullptr;

@@ -52,7 +52,8 @@ class gtr_xs_tables(C.Structure):
                 ("max_num_nucs", C.c_int32), ("egrid", C.c_void_p), ("index_grid", C.c_void_p),
                 ("grid", C.c_void_p), ("num_nucs", C.c_void_p), ("mats", C.c_void_p),
                 ("concs", C.c_void_p), ("grid_type", C.c_int32), ("hash_bins", C.c_int32),
-                ("hash_index", C.c_void_p), ("energies", C.c_void_p)]
+                ("hash_index", C.c_void_p), ("energies", C.c_void_p),
+                ("union_bins", C.c_void_p), ("union_bins_log2", C.c_int32)]
 
 
 XS_UNIONIZED, XS_NUCLIDE, XS_HASH = 0, 1, 2
@@ -100,6 +101,7 @@ _proto = {
     "gtr_xs_build_index_grid": (_i, [_vp, _vp, _i64, _i64, _vp, _vp, _vp, _vp]),
     "gtr_xs_build_energies": (_i, [_vp, _vp, _i64, _i64, _vp, _vp]),
     "gtr_xs_build_hash_grid": (_i, [_vp, _vp, _i64, _i64, C.c_int32, _vp, _vp]),
+    "gtr_xs_build_union_bins": (_i, [_vp, _vp, _i64, C.c_int32, _vp, _vp]),
     "gtr_xs_lookup": (_i, [_vp, _P(gtr_launch_cfg), _P(gtr_xs_tables), _u64, _u64, _u64, _vp,
                            _P(gtr_xs_verify), _vp]),
     "gtr_xs_sorted_workspace_bytes": (_u64, [_u64]),
@@ -213,6 +215,11 @@ def gtr_xs_build_hash_grid(ctx, d_energies, n_iso, n_gp, hash_bins, d_hash_out, 
     return _check("gtr_xs_build_hash_grid", _lib.gtr_xs_build_hash_grid(ctx, _ptr(d_energies), n_iso, n_gp,
                                                                         hash_bins, _ptr(d_hash_out),
                                                                         _stream(stream)))
+
+
+def gtr_xs_build_union_bins(ctx, d_egrid, n_union, log2_bins, d_bins_out, stream=None):
+    return _check("gtr_xs_build_union_bins", _lib.gtr_xs_build_union_bins(ctx, _ptr(d_egrid), n_union, log2_bins,
+                                                                          _ptr(d_bins_out), _stream(stream)))
 
 
 def gtr_xs_build_index_grid(ctx, d_grid, n_iso, n_gp, d_egrid, d_index_out, d_workspace, stream=None):

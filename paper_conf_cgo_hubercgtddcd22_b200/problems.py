@@ -16,9 +16,13 @@ class XsDevice:
     """XS tables on the GPU: the nuclide grid (uploaded) and the acceleration
     structure of `grid_type`, built by libgtr: unionized energy grid + index
     grid (gtr_xs_build_egrid / _index_grid), or the compact per-nuclide
-    energies (+ the hash grid) for the nuclide / hash grid types."""
+    energies (+ the hash grid) for the nuclide / hash grid types.
 
-    def __init__(self, ctx, t, device="cuda", stream=None, grid_type=0, hash_bins=10000):
+    `union_bins_log2` (identical results, on by
+    default): a bin table narrowing the union search (None: the plain
+    full-range binary search)."""
+
+    def __init__(self, ctx, t, device="cuda", stream=None, grid_type=0, hash_bins=10000, union_bins_log2=21):
         self.n_iso, self.n_gp = int(t["n_iso"]), int(t["n_gp"])
         self.n_union = self.n_iso * self.n_gp
         self.grid_type, self.hash_bins = grid_type, hash_bins
@@ -44,17 +48,23 @@ class XsDevice:
                 self.hash_index = torch.empty((hash_bins, self.n_iso), dtype=torch.int32, device=device)
                 G.gtr_xs_build_hash_grid(ctx, self.energies, self.n_iso, self.n_gp, hash_bins, self.hash_index,
                                          stream)
+        self.union_bins, self.union_bins_log2 = None, 0
+        if grid_type == G.XS_UNIONIZED and union_bins_log2 is not None:
+            self.union_bins_log2 = int(union_bins_log2)
+            self.union_bins = torch.empty((1 << self.union_bins_log2) + 1, dtype=torch.int32, device=device)
+            G.gtr_xs_build_union_bins(ctx, self.egrid, self.n_union, self.union_bins_log2, self.union_bins, stream)
         G.gtr_ctx_check(ctx, stream)           # duplicate energies -> GtrError
         p = lambda x: x.data_ptr() if x is not None else None   # noqa: E731
         self.tables = G.gtr_xs_tables(self.n_iso, self.n_gp, self.n_union, self.max_num_nucs,
                                       p(self.egrid), p(self.index_grid), self.grid.data_ptr(),
                                       self.num_nucs.data_ptr(), self.mats.data_ptr(), self.concs.data_ptr(),
-                                      grid_type, hash_bins, p(self.hash_index), p(self.energies))
+                                      grid_type, hash_bins, p(self.hash_index), p(self.energies),
+                                      p(self.union_bins), self.union_bins_log2)
 
     def nbytes(self):
         return sum(x.numel() * x.element_size() for x in
                    (self.grid, self.egrid, self.index_grid, self.energies, self.hash_index, self.num_nucs,
-                    self.mats, self.concs) if x is not None)
+                    self.mats, self.concs, self.union_bins) if x is not None)
 
     def verify_buffers(self, n, device="cuda"):
         bufs = {"mat": torch.zeros(n, dtype=torch.uint8, device=device),

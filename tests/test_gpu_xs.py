@@ -37,6 +37,64 @@ def test_unionized_grid_matches_oracle(dev_small, small):
     assert np.array_equal(dev_small.index_grid.cpu().numpy(), P.index_grid)
 
 
+def test_union_bins_builder(G, ctx, dev_small, small):
+    """bins[b] = searchsorted(egrid, b / 2^L, 'left') on the oracle's egrid."""
+    t, P, *_ = small
+    L = dev_small.union_bins_log2
+    want = np.searchsorted(P.egrid, np.arange((1 << L) + 1) / float(1 << L), side="left")
+    assert np.array_equal(dev_small.union_bins.cpu().numpy().astype(np.int64), want)
+
+
+@pytest.fixture(scope="module")
+def dev_small_plain(G, ctx, small):
+    """Tables without the union bins: the full-range binary search."""
+    from paper_conf_cgo_hubercgtddcd22_b200.problems import XsDevice
+    return XsDevice(ctx, small[0], union_bins_log2=None)
+
+
+@pytest.mark.parametrize("sched", (0, 4), ids=("bucketed", "plain"))
+@pytest.mark.parametrize("variant", [(m, p, f, nt) for m in (0, 1, 2, 3) for p, f in ((3, 1), (0, 0))
+                                     for nt in (128, 256)], ids=vid)
+def test_plain_tables_bit_exact(G, ctx, dev_small_plain, small, variant, sched):
+    t, P, o_out, o_v, n = small
+    m, p, f, nt = variant
+    out, v = _run(G, ctx, dev_small_plain, G.cfg(m, p, f, nt, flags=sched), 0, n)
+    _assert_same(out, v, o_out, o_v)
+    out, v = _run(G, ctx, dev_small_plain, G.cfg(G.NATIVE, G.PL_STACK, 1, nt), 0, n)
+    _assert_same(out, v, o_out, o_v)
+
+
+@pytest.mark.parametrize("log2b", (0, 1, 7, 26))
+def test_union_bins_extreme_sizes(G, ctx, small, log2b):
+    """One bin (the full range), a few, and 2^26 bins (mostly empty, every
+    non-empty bin holds one energy): same results."""
+    from paper_conf_cgo_hubercgtddcd22_b200.problems import XsDevice
+    t, P, o_out, o_v, n = small
+    dev = XsDevice(ctx, t, union_bins_log2=log2b)
+    for mode in (G.SPMD, G.NATIVE):
+        out, v = _run(G, ctx, dev, G.cfg(mode, G.PL_STACK, 1, 256), 0, 20000)
+        _assert_same(out, v, *P.run(0, 20000, X.SEED_L, 4, verify=True))
+
+
+@pytest.mark.parametrize("log2b", (None, 0, 3, 21))
+def test_energies_outside_the_grid(G, ctx, orc, log2b):
+    """Gridpoint energies squeezed into [0.25, 0.75): lookups with E below the
+    first union energy (u = 0) and above the last (u = n_union - 2, the
+    clamp), through every search path."""
+    from paper_conf_cgo_hubercgtddcd22_b200.problems import XsDevice
+    t = X.make_tables(68, 2000)
+    t["grid"][:, :, 0] = 0.25 + 0.5 * t["grid"][:, :, 0]
+    P = orc.XsProblem(t)
+    n = 30000
+    o_out, o_v = P.run(0, n, X.SEED_L, 4, verify=True)
+    assert (o_v["u"] == 0).sum() > 1000 and (o_v["u"] == P.n_union - 2).sum() > 1000
+    dev = XsDevice(ctx, t, union_bins_log2=log2b)
+    for c in (G.cfg(G.SPMD, G.PL_STACK, 1, 256), G.cfg(G.NATIVE, G.PL_STACK, 1, 256),
+              G.cfg(G.GENERIC, G.PL_RUNTIME, 0, 128), G.cfg(G.CSM, G.PL_STACK, 1, 128, flags=G.F_PLAIN)):
+        out, v = _run(G, ctx, dev, c, 0, n)
+        _assert_same(out, v, o_out, o_v)
+
+
 def _run(G, ctx, dev, cfg, first, n, verify=True):
     out = torch.zeros(18, dtype=torch.uint64, device="cuda")
     v, bufs = dev.verify_buffers(n) if verify else (None, None)

@@ -43,9 +43,10 @@ ap.add_argument("--niso", type=int, default=355)
 ap.add_argument("--time", action="store_true")
 ap.add_argument("--persist", type=float, default=0.0, help="L2 persisting window over the grid, hit ratio")
 ap.add_argument("--persist-mb", type=int, default=96)
+ap.add_argument("--bins", type=int, default=21, help="log2 union bins; -1: full-range union search")
 a = ap.parse_args()
 ctx = G.gtr_ctx_create(0)
-xs = XsDevice(ctx, X.make_tables(a.niso))
+xs = XsDevice(ctx, X.make_tables(a.niso), union_bins_log2=None if a.bins < 0 else a.bins)
 out = torch.zeros(18, dtype=torch.uint64, device="cuda")
 if a.persist > 0:
     G.gtr_l2_persist(ctx, xs.grid, xs.grid.numel() * 8, a.persist_mb << 20, a.persist)
