@@ -77,8 +77,13 @@ __device__ __forceinline__ cx fast_cexp(cx z) {
 // per pole, each an XU-pipe reciprocal plus a Newton sequence; the XU pipe
 // was the busiest unit (ncu: 75% of peak).  |Z| < 6 is tested as |Z|^2 < 36
 // (same branch: sqrt is monotonic and correctly rounded).
-__device__ __forceinline__ cx faddeeva(cx Z) {
-    if (Z.r * Z.r + Z.i * Z.i < 36.0) {
+#ifndef GTR_RS_POLES2
+#define GTR_RS_POLES2 0
+#endif
+constexpr int kPolesPerStep = GTR_RS_POLES2 ? 2 : 1;
+__device__ __forceinline__ bool faddeeva_inner_branch(cx Z) { return Z.r * Z.r + Z.i * Z.i < 36.0; }
+__device__ __forceinline__ cx faddeeva_series(cx Z) {
+    {
         constexpr double an[10] = {2.758402e-01, 2.245740e-01, 1.594149e-01, 9.866577e-02, 5.324414e-02,
                                    2.505215e-02, 1.027747e-02, 3.676164e-03, 1.146494e-03, 3.117570e-04};
         constexpr double dl[10] = {9.869604e+00, 3.947842e+01, 8.882644e+01, 1.579137e+02, 2.467401e+02,
@@ -112,6 +117,9 @@ __device__ __forceinline__ cx faddeeva(cx Z) {
         const cx zs = cmul(Z, sum);
         return {W0.r - 8.124330e+01 * zs.i, W0.i + 8.124330e+01 * zs.r};   // W0 + i 81.2433 Z sum
     }
+}
+__device__ __forceinline__ cx faddeeva(cx Z) {
+    if (faddeeva_inner_branch(Z)) return faddeeva_series(Z);
     const cx a = {0.512424224754768462984202823134979415014943561548661637413182, 0.0};
     const cx b = {0.275255128608410950901357962647054304017026259671664935783653, 0.0};
     const cx c = {0.051765358792987823963876628425793170829107067780337219430904, 0.0};
@@ -133,8 +141,8 @@ struct TagSig {};
 template <class K, class LM>
 __device__ __forceinline__ void micro_xs(const Params &P, int64_t nuc, double E, LM &micro) {
     Local<K, double, 8, TagSigTF> sf;     // sigTfactors[4] complex
-    Local<K, double, 2, TagZ> Zv;
-    Local<K, double, 2, TagW> Wv;
+    Local<K, double, 2 * kPolesPerStep, TagZ> Zv;
+    Local<K, double, 2 * kPolesPerStep, TagW> Wv;
     Local<K, double, 3, TagSig> sig;
     const int32_t nw = __ldg(P.n_windows + nuc);
     const double spacing = 1.0 / nw;
@@ -158,7 +166,45 @@ __device__ __forceinline__ void micro_xs(const Params &P, int64_t nuc, double E,
     sig[0] = E * __ldg(w + 0);
     sig[1] = E * __ldg(w + 1);
     sig[2] = E * __ldg(w + 2);
-    for (int32_t p = se.x; p < se.y; p++) {
+    int32_t p = se.x;
+#if GTR_RS_POLES2
+    // two poles per iteration: both Faddeeva evaluations in straight-line
+    // code (when both take the series branch, always for |Z| < 6) so their
+    // dependency chains interleave; accumulation stays in pole order
+    for (; p + 1 < se.y; p += 2) {
+        const double *pr = P.poles + (nuc * P.max_poles + p) * 9;
+        const double *pq = pr + 9;
+        const cx Z1 = cmul(csub(cx{E, 0.0}, cx{__ldg(pr + 0), __ldg(pr + 1)}), cx{0.5, 0.0});
+        const cx Z2 = cmul(csub(cx{E, 0.0}, cx{__ldg(pq + 0), __ldg(pq + 1)}), cx{0.5, 0.0});
+        Zv[0] = Z1.r;
+        Zv[1] = Z1.i;
+        Zv[2] = Z2.r;
+        Zv[3] = Z2.i;
+        cx W1, W2;
+        if (faddeeva_inner_branch(cx{Zv[0], Zv[1]}) && faddeeva_inner_branch(cx{Zv[2], Zv[3]})) {
+            W1 = faddeeva_series(cx{Zv[0], Zv[1]});
+            W2 = faddeeva_series(cx{Zv[2], Zv[3]});
+        } else {
+            W1 = faddeeva(cx{Zv[0], Zv[1]});
+            W2 = faddeeva(cx{Zv[2], Zv[3]});
+        }
+        Wv[0] = W1.r;
+        Wv[1] = W1.i;
+        Wv[2] = W2.r;
+        Wv[3] = W2.i;
+#pragma unroll
+        for (int q = 0; q < 2; q++) {
+            const double *pp = q ? pq : pr;
+            const cx Wl = {Wv[2 * q], Wv[2 * q + 1]};
+            const int lv = __ldg(reinterpret_cast<const int *>(pp + 8));
+            const cx f = {sf[2 * lv], sf[2 * lv + 1]};
+            sig[0] = sig[0] + cmul(cx{__ldg(pp + 2), __ldg(pp + 3)}, cmul(Wl, f)).r;
+            sig[1] = sig[1] + cmul(cx{__ldg(pp + 4), __ldg(pp + 5)}, Wl).r;
+            sig[2] = sig[2] + cmul(cx{__ldg(pp + 6), __ldg(pp + 7)}, Wl).r;
+        }
+    }
+#endif
+    for (; p < se.y; p++) {
         const double *pr = P.poles + (nuc * P.max_poles + p) * 9;
         // 72-byte records: 8-byte aligned only, so scalar loads
         const double2 EA = make_double2(__ldg(pr + 0), __ldg(pr + 1));
