@@ -65,6 +65,8 @@ static rs::Params make_params(const gtr_rs_tables *t, uint64_t first, uint64_t n
         P.num_nucs = t->num_nucs;
         P.mats = t->mats;
         P.concs = t->concs;
+        P.poles_wide = t->poles_wide;
+        P.wide = ((reinterpret_cast<uintptr_t>(t->windows) | reinterpret_cast<uintptr_t>(t->k0rs)) & 31u) == 0;
         P.n_nuc = t->n_nuc;
         P.max_poles = t->max_poles;
         P.max_windows = t->max_windows;
@@ -85,11 +87,36 @@ int gtr_internal_query_rs(gtr_ctx *ctx, const gtr_launch_cfg *cfg, gtr_variant_i
     return rs::launch(a);
 }
 
+namespace gtr {
+namespace rs {
+__global__ void k_wide_poles(const double *__restrict__ poles, int64_t n_rec, double *__restrict__ out) {
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n_rec * 12;
+         i += (int64_t)gridDim.x * blockDim.x) {
+        const int64_t r = i / 12, w = i - r * 12;
+        out[i] = w < 9 ? __ldg(poles + r * 9 + w) : 0.0;
+    }
+}
+}  // namespace rs
+}  // namespace gtr
+
+extern "C" int gtr_rs_build_wide_poles(gtr_ctx *ctx, const double *d_poles, int64_t n_records,
+                                       double *d_poles_wide_out, void *stream) {
+    if (!ctx || !d_poles || !d_poles_wide_out || n_records < 1 ||
+        (reinterpret_cast<uintptr_t>(d_poles_wide_out) & 31u))
+        return GTR_EINVAL;
+    const int64_t blocks = (n_records * 12 + 255) / 256, cap = (int64_t)ctx->num_sms * 16;
+    rs::k_wide_poles<<<(int)(blocks < cap ? blocks : cap), 256, 0, static_cast<cudaStream_t>(stream)>>>(
+        d_poles, n_records, d_poles_wide_out);
+    GTR_CUDA_TRY(cudaGetLastError());
+    return GTR_OK;
+}
+
 extern "C" int gtr_rs_lookup(gtr_ctx *ctx, const gtr_launch_cfg *cfg, const gtr_rs_tables *t, uint64_t first,
                              uint64_t n, uint64_t seed, uint64_t *d_out, const gtr_rs_verify *verify,
                              void *stream) {
     if (!ctx || !cfg || !t || !d_out || !t->n_windows || !t->poles || !t->windows || !t->k0rs ||
-        !t->num_nucs || !t->mats || !t->concs || t->n_nuc < 1 || t->max_poles < 1 || t->max_windows < 1)
+        !t->num_nucs || !t->mats || !t->concs || t->n_nuc < 1 || t->max_poles < 1 || t->max_windows < 1 ||
+        (reinterpret_cast<uintptr_t>(t->poles_wide) & 31u))
         return GTR_EINVAL;
     if (n == 0) return GTR_OK;
     rs::LaunchArgs a{ctx, cfg, make_params(t, first, n, seed, d_out, verify), static_cast<cudaStream_t>(stream),

@@ -27,6 +27,8 @@ struct Params {
     const int32_t *num_nucs;
     const int32_t *mats;
     const double *concs;
+    const double *poles_wide; // 12 words per record, 32-byte aligned, or null
+    int32_t wide;             // windows and k0rs 32-byte aligned: 256-bit loads
     int64_t n_nuc, max_poles, max_windows;
     int32_t max_num_nucs;
     uint32_t chunk;
@@ -50,6 +52,13 @@ __device__ __forceinline__ cx cdiv(cx a, cx b) {
     return {((a.r * b.r) + (a.i * b.i)) / d, ((a.i * b.r) - (a.r * b.i)) / d};
 }
 __device__ __forceinline__ double cabs_(cx a) { return sqrt(a.r * a.r + a.i * a.i); }
+
+#ifndef GTR_RS_PREFETCH
+#define GTR_RS_PREFETCH 1
+#endif
+__device__ __forceinline__ void ld256(const double *a, double &x0, double &x1, double &x2, double &x3) {
+    asm("ld.global.nc.v4.f64 {%0, %1, %2, %3}, [%4];" : "=d"(x0), "=d"(x1), "=d"(x2), "=d"(x3) : "l"(a));
+}
 
 __device__ __forceinline__ double fast_exp(double x) {
     x = 1.0 + x * 0.000244140625;
@@ -77,10 +86,6 @@ __device__ __forceinline__ cx fast_cexp(cx z) {
 // per pole, each an XU-pipe reciprocal plus a Newton sequence; the XU pipe
 // was the busiest unit (ncu: 75% of peak).  |Z| < 6 is tested as |Z|^2 < 36
 // (same branch: sqrt is monotonic and correctly rounded).
-#ifndef GTR_RS_POLES2
-#define GTR_RS_POLES2 0
-#endif
-constexpr int kPolesPerStep = GTR_RS_POLES2 ? 2 : 1;
 __device__ __forceinline__ bool faddeeva_inner_branch(cx Z) { return Z.r * Z.r + Z.i * Z.i < 36.0; }
 __device__ __forceinline__ cx faddeeva_series(cx Z) {
     {
@@ -141,17 +146,24 @@ struct TagSig {};
 template <class K, class LM>
 __device__ __forceinline__ void micro_xs(const Params &P, int64_t nuc, double E, LM &micro) {
     Local<K, double, 8, TagSigTF> sf;     // sigTfactors[4] complex
-    Local<K, double, 2 * kPolesPerStep, TagZ> Zv;
-    Local<K, double, 2 * kPolesPerStep, TagW> Wv;
+    Local<K, double, 2, TagZ> Zv;
+    Local<K, double, 2, TagW> Wv;
     Local<K, double, 3, TagSig> sig;
     const int32_t nw = __ldg(P.n_windows + nuc);
     const double spacing = 1.0 / nw;
     int32_t window = (int32_t)(E / spacing);
     if (window == nw) window--;
     const double sqE = sqrt(E);
+    double k0[4];
+    if (P.wide) {
+        ld256(P.k0rs + nuc * 4, k0[0], k0[1], k0[2], k0[3]);
+    } else {
+#pragma unroll
+        for (int l = 0; l < 4; l++) k0[l] = __ldg(P.k0rs + nuc * 4 + l);
+    }
 #pragma unroll
     for (int l = 0; l < 4; l++) {
-        double phi = __ldg(P.k0rs + nuc * 4 + l) * sqE;
+        double phi = k0[l] * sqE;
         if (l == 1) phi -= -atan(phi);
         else if (l == 2) phi -= atan(3.0 * phi / (3.0 - phi * phi));
         else if (l == 3) phi -= atan(phi * (15.0 - phi * phi) / (15.0 - 6.0 * phi * phi));
@@ -162,56 +174,21 @@ __device__ __forceinline__ void micro_xs(const Params &P, int64_t nuc, double E,
         sf[2 * l + 1] = -s;
     }
     const double *w = P.windows + (nuc * P.max_windows + window) * 4;
-    const int2 se = *reinterpret_cast<const int2 *>(w + 3);
-    sig[0] = E * __ldg(w + 0);
-    sig[1] = E * __ldg(w + 1);
-    sig[2] = E * __ldg(w + 2);
-    int32_t p = se.x;
-#if GTR_RS_POLES2
-    // two poles per iteration: both Faddeeva evaluations in straight-line
-    // code (when both take the series branch, always for |Z| < 6) so their
-    // dependency chains interleave; accumulation stays in pole order
-    for (; p + 1 < se.y; p += 2) {
-        const double *pr = P.poles + (nuc * P.max_poles + p) * 9;
-        const double *pq = pr + 9;
-        const cx Z1 = cmul(csub(cx{E, 0.0}, cx{__ldg(pr + 0), __ldg(pr + 1)}), cx{0.5, 0.0});
-        const cx Z2 = cmul(csub(cx{E, 0.0}, cx{__ldg(pq + 0), __ldg(pq + 1)}), cx{0.5, 0.0});
-        Zv[0] = Z1.r;
-        Zv[1] = Z1.i;
-        Zv[2] = Z2.r;
-        Zv[3] = Z2.i;
-        cx W1, W2;
-        if (faddeeva_inner_branch(cx{Zv[0], Zv[1]}) && faddeeva_inner_branch(cx{Zv[2], Zv[3]})) {
-            W1 = faddeeva_series(cx{Zv[0], Zv[1]});
-            W2 = faddeeva_series(cx{Zv[2], Zv[3]});
-        } else {
-            W1 = faddeeva(cx{Zv[0], Zv[1]});
-            W2 = faddeeva(cx{Zv[2], Zv[3]});
-        }
-        Wv[0] = W1.r;
-        Wv[1] = W1.i;
-        Wv[2] = W2.r;
-        Wv[3] = W2.i;
-#pragma unroll
-        for (int q = 0; q < 2; q++) {
-            const double *pp = q ? pq : pr;
-            const cx Wl = {Wv[2 * q], Wv[2 * q + 1]};
-            const int lv = __ldg(reinterpret_cast<const int *>(pp + 8));
-            const cx f = {sf[2 * lv], sf[2 * lv + 1]};
-            sig[0] = sig[0] + cmul(cx{__ldg(pp + 2), __ldg(pp + 3)}, cmul(Wl, f)).r;
-            sig[1] = sig[1] + cmul(cx{__ldg(pp + 4), __ldg(pp + 5)}, Wl).r;
-            sig[2] = sig[2] + cmul(cx{__ldg(pp + 6), __ldg(pp + 7)}, Wl).r;
-        }
+    double wT, wA, wF, wse;
+    if (P.wide) {                                    // one 32-byte record, one sector
+        ld256(w, wT, wA, wF, wse);
+    } else {
+        wT = __ldg(w + 0);
+        wA = __ldg(w + 1);
+        wF = __ldg(w + 2);
+        wse = __ldg(w + 3);
     }
-#endif
-    for (; p < se.y; p++) {
-        const double *pr = P.poles + (nuc * P.max_poles + p) * 9;
-        // 72-byte records: 8-byte aligned only, so scalar loads
-        const double2 EA = make_double2(__ldg(pr + 0), __ldg(pr + 1));
-        const double2 RT = make_double2(__ldg(pr + 2), __ldg(pr + 3));
-        const double2 RA = make_double2(__ldg(pr + 4), __ldg(pr + 5));
-        const double2 RF = make_double2(__ldg(pr + 6), __ldg(pr + 7));
-        const int lv = __ldg(reinterpret_cast<const int *>(pr + 8));
+    const int2 se = make_int2(__double2loint(wse), __double2hiint(wse));
+    sig[0] = E * wT;
+    sig[1] = E * wA;
+    sig[2] = E * wF;
+    // one pole (c4 step 4), in pole order
+    auto pole = [&](double2 EA, double2 RT, double2 RA, double2 RF, int lv) {
         const cx Z = cmul(csub(cx{E, 0.0}, cx{EA.x, EA.y}), cx{0.5, 0.0});
         Zv[0] = Z.r;
         Zv[1] = Z.i;
@@ -223,6 +200,41 @@ __device__ __forceinline__ void micro_xs(const Params &P, int64_t nuc, double E,
         sig[0] = sig[0] + cmul(cx{RT.x, RT.y}, cmul(Wl, f)).r;
         sig[1] = sig[1] + cmul(cx{RA.x, RA.y}, Wl).r;
         sig[2] = sig[2] + cmul(cx{RF.x, RF.y}, Wl).r;
+    };
+    if (P.poles_wide) {
+        // 96-byte records: 2 x 256 bit + the l word
+        const double *base = P.poles_wide + nuc * P.max_poles * 12;
+#if GTR_RS_PREFETCH
+        // the next pole's first 32 bytes (EA, RT) are loaded before this
+        // pole's Faddeeva evaluation: the load that starts each pole is
+        // already in flight
+        double2 nEA = {0.0, 0.0}, nRT = {0.0, 0.0};
+        if (se.x < se.y) ld256(base + (int64_t)se.x * 12, nEA.x, nEA.y, nRT.x, nRT.y);
+        for (int32_t p = se.x; p < se.y; p++) {
+            const double *pr = base + (int64_t)p * 12;
+            const double2 EA = nEA, RT = nRT;
+            double2 RA, RF;
+            ld256(pr + 4, RA.x, RA.y, RF.x, RF.y);
+            const int lv = __ldg(reinterpret_cast<const int *>(pr + 8));
+            if (p + 1 < se.y) ld256(pr + 12, nEA.x, nEA.y, nRT.x, nRT.y);
+            pole(EA, RT, RA, RF, lv);
+        }
+#else
+        for (int32_t p = se.x; p < se.y; p++) {
+            const double *pr = base + (int64_t)p * 12;
+            double2 EA, RT, RA, RF;
+            ld256(pr + 0, EA.x, EA.y, RT.x, RT.y);
+            ld256(pr + 4, RA.x, RA.y, RF.x, RF.y);
+            pole(EA, RT, RA, RF, __ldg(reinterpret_cast<const int *>(pr + 8)));
+        }
+#endif
+    } else {
+        for (int32_t p = se.x; p < se.y; p++) {      // 72-byte records: 8-byte aligned only, scalar loads
+            const double *pr = P.poles + (nuc * P.max_poles + p) * 9;
+            pole(make_double2(__ldg(pr + 0), __ldg(pr + 1)), make_double2(__ldg(pr + 2), __ldg(pr + 3)),
+                 make_double2(__ldg(pr + 4), __ldg(pr + 5)), make_double2(__ldg(pr + 6), __ldg(pr + 7)),
+                 __ldg(reinterpret_cast<const int *>(pr + 8)));
+        }
     }
     micro[0] = sig[0];
     micro[1] = sig[1];

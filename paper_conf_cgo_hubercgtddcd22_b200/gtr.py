@@ -71,7 +71,7 @@ class gtr_rs_tables(C.Structure):
     _fields_ = [("n_nuc", C.c_int64), ("max_poles", C.c_int64), ("max_windows", C.c_int64),
                 ("max_num_nucs", C.c_int32), ("n_windows", C.c_void_p), ("poles", C.c_void_p),
                 ("windows", C.c_void_p), ("k0rs", C.c_void_p), ("num_nucs", C.c_void_p),
-                ("mats", C.c_void_p), ("concs", C.c_void_p)]
+                ("mats", C.c_void_p), ("concs", C.c_void_p), ("poles_wide", C.c_void_p)]
 
 
 class gtr_rs_verify(C.Structure):
@@ -102,6 +102,7 @@ _proto = {
     "gtr_xs_build_energies": (_i, [_vp, _vp, _i64, _i64, _vp, _vp]),
     "gtr_xs_build_hash_grid": (_i, [_vp, _vp, _i64, _i64, C.c_int32, _vp, _vp]),
     "gtr_xs_build_union_bins": (_i, [_vp, _vp, _i64, C.c_int32, _vp, _vp]),
+    "gtr_rs_build_wide_poles": (_i, [_vp, _vp, _i64, _vp, _vp]),
     "gtr_xs_lookup": (_i, [_vp, _P(gtr_launch_cfg), _P(gtr_xs_tables), _u64, _u64, _u64, _vp,
                            _P(gtr_xs_verify), _vp]),
     "gtr_xs_sorted_workspace_bytes": (_u64, [_u64]),
@@ -220,6 +221,11 @@ def gtr_xs_build_hash_grid(ctx, d_energies, n_iso, n_gp, hash_bins, d_hash_out, 
 def gtr_xs_build_union_bins(ctx, d_egrid, n_union, log2_bins, d_bins_out, stream=None):
     return _check("gtr_xs_build_union_bins", _lib.gtr_xs_build_union_bins(ctx, _ptr(d_egrid), n_union, log2_bins,
                                                                           _ptr(d_bins_out), _stream(stream)))
+
+
+def gtr_rs_build_wide_poles(ctx, d_poles, n_records, d_out, stream=None):
+    return _check("gtr_rs_build_wide_poles", _lib.gtr_rs_build_wide_poles(ctx, _ptr(d_poles), n_records, _ptr(d_out),
+                                                                          _stream(stream)))
 
 
 def gtr_xs_build_index_grid(ctx, d_grid, n_iso, n_gp, d_egrid, d_index_out, d_workspace, stream=None):

@@ -77,7 +77,11 @@ class XsDevice:
 
 
 class RsDevice:
-    def __init__(self, t, device="cuda"):
+    """RS tables on the GPU.  `wide_poles` (on by default; identical results):
+    also build the 96-byte pole records (gtr_rs_build_wide_poles) the lookups
+    then read with 256-bit loads; False keeps RSBench's 72-byte records."""
+
+    def __init__(self, t, device="cuda", ctx=None, wide_poles=True, stream=None):
         self.n_windows = _dev(t["n_windows"].astype(np.int32), device)
         self.poles = _dev(np.ascontiguousarray(t["poles"]).view(np.uint8), device)
         self.windows = _dev(np.ascontiguousarray(t["windows"]).view(np.uint8), device)
@@ -85,10 +89,21 @@ class RsDevice:
         self.num_nucs = _dev(t["num_nucs"].astype(np.int32), device)
         self.mats = _dev(t["mats"].astype(np.int32), device)
         self.concs = _dev(t["concs"].astype(np.float64), device)
+        self.poles_wide = None
+        if wide_poles:
+            own = ctx is None
+            c = G.gtr_ctx_create(torch.device(device).index or 0) if own else ctx
+            n_rec = int(t["n_nuc"]) * int(t["max_poles"])
+            self.poles_wide = torch.empty((n_rec, 12), dtype=torch.float64, device=device)
+            G.gtr_rs_build_wide_poles(c, self.poles, n_rec, self.poles_wide, stream)
+            G.gtr_ctx_check(c, stream)
+            if own:
+                G.gtr_ctx_destroy(c)
         self.tables = G.gtr_rs_tables(int(t["n_nuc"]), int(t["max_poles"]), int(t["max_windows"]),
                                       int(t["mats"].shape[1]), self.n_windows.data_ptr(), self.poles.data_ptr(),
                                       self.windows.data_ptr(), self.k0rs.data_ptr(), self.num_nucs.data_ptr(),
-                                      self.mats.data_ptr(), self.concs.data_ptr())
+                                      self.mats.data_ptr(), self.concs.data_ptr(),
+                                      self.poles_wide.data_ptr() if self.poles_wide is not None else None)
 
     def verify_buffers(self, n, device="cuda"):
         bufs = {"mat": torch.zeros(n, dtype=torch.uint8, device=device),

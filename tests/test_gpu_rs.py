@@ -58,3 +58,36 @@ def test_rs_all_variants(G, ctx, dev, rs, variant, sched):
 @pytest.mark.parametrize("nt", (128, 256))
 def test_rs_native(G, ctx, dev, rs, nt):
     _check(G, ctx, dev, rs, G.cfg(G.NATIVE, G.PL_STACK, 1, nt))
+
+
+@pytest.fixture(scope="module")
+def dev_narrow(rs):
+    """RSBench's 72-byte pole records (no wide-pole table)."""
+    from paper_conf_cgo_hubercgtddcd22_b200.problems import RsDevice
+    return RsDevice(rs[0], wide_poles=False)
+
+
+def test_rs_wide_poles_builder(dev, rs):
+    """poles_wide[r] = the 72-byte record's 9 words + 3 zero words."""
+    t = rs[0]
+    raw = np.ascontiguousarray(t["poles"]).view(np.float64).reshape(-1, 9)
+    got = dev.poles_wide.cpu().numpy()
+    assert np.array_equal(got[:, :9].view(np.uint64), raw.view(np.uint64))
+    assert (got[:, 9:] == 0).all()
+
+
+@pytest.mark.parametrize("cfg", [(0, 0, 0, 128), (2, 3, 1, 128), (3, 3, 1, 128), (3, 0, 0, 128), (4, 3, 1, 128),
+                                 (4, 3, 1, 256)], ids=lambda v: "m%d-p%d-f%d-t%d" % v)
+def test_rs_narrow_records(G, ctx, dev_narrow, rs, cfg):
+    m, p, f, nt = cfg
+    _check(G, ctx, dev_narrow, rs, G.cfg(m, p, f, nt))
+
+
+def test_rs_wide_poles_misaligned_rejected(G, ctx, dev, rs):
+    import ctypes
+    t = G.gtr_rs_tables.from_buffer_copy(dev.tables)
+    t.poles_wide = dev.poles_wide.data_ptr() + 8
+    out = torch.zeros(18, dtype=torch.uint64, device="cuda")
+    with pytest.raises(G.GtrError):
+        G.gtr_rs_lookup(ctx, G.cfg(G.SPMD, G.PL_STACK, 1, 128), t, 0, 10, X.SEED_L, out)
+    assert ctypes.sizeof(t) == ctypes.sizeof(dev.tables)

@@ -29,9 +29,10 @@ ap.add_argument("variants", nargs="+")
 ap.add_argument("--n", type=int, default=200_000)
 ap.add_argument("--reps", type=int, default=1)
 ap.add_argument("--time", action="store_true")
+ap.add_argument("--narrow", action="store_true", help="RSBench's 72-byte pole records")
 a = ap.parse_args()
 ctx = G.gtr_ctx_create(0)
-rs = RsDevice(RS.make_tables())
+rs = RsDevice(RS.make_tables(), ctx=ctx, wide_poles=not a.narrow)
 out = torch.zeros(18, dtype=torch.uint64, device="cuda")
 for v in a.variants:
     c = VARIANTS[v]
