@@ -91,3 +91,36 @@ def test_rs_wide_poles_misaligned_rejected(G, ctx, dev, rs):
     with pytest.raises(G.GtrError):
         G.gtr_rs_lookup(ctx, G.cfg(G.SPMD, G.PL_STACK, 1, 128), t, 0, 10, X.SEED_L, out)
     assert ctypes.sizeof(t) == ctypes.sizeof(dev.tables)
+
+
+@pytest.mark.slow
+def test_rs_full_size_bench_launch(G, ctx, orc):
+    """Config 4 at full size (355 nuclides, 10M lookups) in the launch
+    configuration bench.py times (SPMD + heap-to-stack + folding, thread
+    limit 128, wide pole records): the whole run's tallies are consistent
+    (every lookup counted once, hash = sum (argmax+1) x tally), and five
+    ranges of 3000 lookups spread over [0, 10M) match the oracle element by
+    element (R-RS-tol) with identical materials and argmaxes."""
+    import os
+    from paper_conf_cgo_hubercgtddcd22_b200.problems import RsDevice
+    t = RS.make_tables()
+    dev = RsDevice(t, ctx=ctx)
+    n = 10_000_000
+    out = torch.zeros(18, dtype=torch.uint64, device="cuda")
+    v, bufs = dev.verify_buffers(n)
+    G.gtr_rs_lookup(ctx, G.cfg(G.SPMD, G.PL_STACK, 1, 128), dev.tables, 0, n, X.SEED_L, out, v)
+    G.gtr_ctx_check(ctx)
+    res = out.cpu().numpy()
+    assert int(res[1:13].sum()) == n and int(res[13:17].sum()) == n
+    assert int(res[0]) == sum((k + 1) * int(res[13 + k]) for k in range(4))
+    P = orc.RsProblem(t)
+    m = 3000
+    for first in (0, 2_345_678, 5_000_000, 7_777_777, n - m):
+        o_out, o_v, margin = P.run(first, m, X.SEED_L, os.cpu_count() or 8, verify=True)
+        assert margin > 1e-10
+        sl = slice(first, first + m)
+        assert np.array_equal(bufs["mat"][sl].cpu().numpy(), o_v["mat"])
+        assert np.array_equal(bufs["am"][sl].cpu().numpy(), o_v["am"])
+        got, want = bufs["macro"][sl].cpu().numpy(), o_v["macro"]
+        scale = np.abs(want).max(axis=1, keepdims=True)
+        assert (np.abs(got - want) <= 1e-12 * scale).all(), (first, np.abs(got - want).max())
