@@ -37,6 +37,10 @@ for m in modes + (G.NATIVE,):
         out = torch.zeros(18, dtype=torch.uint64, device="cuda")
         G.gtr_xs_lookup(ctx, G.cfg(m, G.PL_STACK if m == G.NATIVE else G.PL_RUNTIME, 0, 128, num_teams=teams,
                                    flags=flags), xs.tables, 0, 3000, X.SEED_L, out)
+for m in (G.CSM, G.SPMD):      # the headline kernels (CSM register-capped), union bins on
+    for nt in (128, 256):
+        out = torch.zeros(18, dtype=torch.uint64, device="cuda")
+        G.gtr_xs_lookup(ctx, G.cfg(m, G.PL_STACK, 1, nt, num_teams=teams), xs.tables, 0, 3000, X.SEED_L, out)
 A, B = S.make_lattice(40, "random")
 dA, dB = su3_device(A, B)
 dC = torch.empty_like(dA)
@@ -46,5 +50,6 @@ rs = RsDevice(RS.make_tables(n_nuc=20, avg_poles=40, avg_windows=5))
 for m in modes:
     out = torch.zeros(18, dtype=torch.uint64, device="cuda")
     G.gtr_rs_lookup(ctx, G.cfg(m, G.PL_RUNTIME, 0, 128, num_teams=teams), rs.tables, 0, 700, X.SEED_L, out)
+    G.gtr_rs_lookup(ctx, G.cfg(m, G.PL_STACK, 1, 128, num_teams=teams), rs.tables, 0, 700, X.SEED_L, out)
 G.gtr_ctx_check(ctx)
 print("sanitize run ok")
