@@ -687,6 +687,13 @@ template <class K, class T, class Tag, bool RO = true> struct TeamLocal {
 };
 
 // ---------------------------------------------------------------- worksharing
+// `teams distribute dist_schedule(static, 1)` over [lo, hi): iteration c goes
+// to team (c - lo) mod num_teams (Fig. 1's outer loop).  The body
+// is the team's sequential code (it may fork parallel regions).
+template <class K, class F> __device__ __forceinline__ void distribute_static(int64_t lo, int64_t hi, F &&body) {
+    for (int64_t c = lo + team_num<K>(); c < hi; c += num_teams<K>()) body(c);
+}
+
 // `for` with a static schedule, chunk 1 (cyclic) -- AMB-2: coalesced.
 template <class K, class F> __device__ __forceinline__ void for_static(int64_t lo, int64_t hi, F &&body) {
     const int64_t t = thread_num<K>(), n = num_threads<K>();

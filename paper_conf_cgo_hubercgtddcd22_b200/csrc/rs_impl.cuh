@@ -384,7 +384,8 @@ template <class K> __global__ void __launch_bounds__(K::BLOCK, K::NT == 128 ? (K
     });
     const uint64_t n = P.n, ch = P.chunk;
     const uint64_t nchunks = (n + ch - 1) / ch;
-    for (uint64_t c = team_num<K>(); c < nchunks; c += num_teams<K>()) {
+    distribute_static<K>(0, (int64_t)nchunks, [&](int64_t ci) {   // teams distribute
+        const uint64_t c = (uint64_t)ci;
         TeamLocal<K, Chunk, TagChunk> chunk;
         chunk.set([&](Chunk &x) {
             x.base = P.first + c * ch;
@@ -392,7 +393,7 @@ template <class K> __global__ void __launch_bounds__(K::BLOCK, K::NT == 128 ? (K
         });
         if (P.plain) {
             parallel<K, LookupRegion<K>>(chunk.get());
-            continue;
+            return;
         }
         ChunkBuf<K> &b = chunk_buf<K>();
         guarded<K>([&] {
@@ -409,7 +410,7 @@ template <class K> __global__ void __launch_bounds__(K::BLOCK, K::NT == 128 ? (K
         });
         parallel<K, ScatterRegion<K>>(chunk.get());
         parallel<K, BucketRegion<K>>(chunk.get());
-    }
+    });
     if constexpr (K::MODE == SPMD) flush(g_tally, g_p.out, threadIdx.x, K::NT);
     else flush(g_tally, g_p.out, 0, 1);
     team_deinit<K>();

@@ -171,11 +171,11 @@ template <class K> __global__ void __launch_bounds__(K::BLOCK) kernel_rt(Params 
         team_deinit<K>();
         return;
     }
-    for (int64_t s = team_num<K>(); s < P.sites; s += num_teams<K>()) {   // teams distribute
+    distribute_static<K>(0, P.sites, [&](int64_t s) {   // teams distribute
         TeamLocal<K, Site, TagSite> site;
         site.set([&](Site &x) { x.s = s; });
         parallel<K, SiteRegion<K>>(site.get());
-    }
+    });
     team_deinit<K>();
 }
 
