@@ -431,9 +431,13 @@ def sweeps(G, torch, ctx, xs, first, seed, stream):
         def f():
             out.zero_()
             G.gtr_xs_lookup(ctx, c, xs.tables, first, n, seed, out, None, stream)
+        G.gtr_ctx_fallback_high_water(ctx, reset=True, stream=stream)
         ms = _time(torch, stream, f, 2)
+        info = G.gtr_query_variant(G.K_XS, c)
         ladder[name] = {"lookups_per_s": n / (ms * 1e-3), "ms": ms,
-                        "same_result": bool(np.array_equal(out.cpu().numpy(), ref))}
+                        "same_result": bool(np.array_equal(out.cpu().numpy(), ref)),
+                        "regs": info["regs"], "static_smem": info["static_smem"], "dyn_smem": info["dyn_smem"],
+                        "fallback_bytes_per_thread": G.gtr_ctx_fallback_high_water(ctx, reset=True, stream=stream)}
     G.gtr_ctx_check(ctx, stream)
     # fork/join ns: 148 teams (one per SM), 20,000 trivial regions, K = 4
     fj = {}
@@ -621,11 +625,13 @@ def rs_sweep(G, torch, ctx, stream, n=10_000_000):
         def f():
             out.zero_()
             G.gtr_rs_lookup(ctx, c, dev.tables, 0, n, X.SEED_L, out, None, stream)
+        G.gtr_ctx_fallback_high_water(ctx, reset=True, stream=stream)
         ms = _time(torch, stream, f, 1)
         r = out.cpu().numpy()
         ref = r if ref is None else ref
         res[name] = {"lookups_per_s": n / (ms * 1e-3), "ms": ms, "regs": G.gtr_query_variant(G.K_RS, c)["regs"],
-                     "same_result": bool(np.array_equal(r, ref))}
+                     "same_result": bool(np.array_equal(r, ref)),
+                     "fallback_bytes_per_thread": G.gtr_ctx_fallback_high_water(ctx, reset=True, stream=stream)}
     G.gtr_ctx_check(ctx, stream)
     res["roofline_spmd"] = rs_roofline(G, torch, ctx, stream, 0, n, res["spmd"]["ms"])
     return res

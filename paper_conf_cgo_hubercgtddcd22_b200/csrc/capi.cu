@@ -67,6 +67,18 @@ extern "C" int gtr_ctx_check(gtr_ctx *c, void *stream) {
     return GTR_EDEVICE;
 }
 
+extern "C" int gtr_ctx_fallback_high_water(gtr_ctx *c, uint64_t *bytes_out, int32_t reset, void *stream) {
+    if (!c || !bytes_out) return GTR_EINVAL;
+    cudaStream_t s = static_cast<cudaStream_t>(stream);
+    unsigned long long *d = reinterpret_cast<unsigned long long *>(reinterpret_cast<char *>(c->d_err) + 8);
+    unsigned long long v = 0;
+    GTR_CUDA_TRY(cudaMemcpyAsync(&v, d, sizeof(v), cudaMemcpyDeviceToHost, s));
+    if (reset) GTR_CUDA_TRY(cudaMemsetAsync(d, 0, sizeof(v), s));
+    GTR_CUDA_TRY(cudaStreamSynchronize(s));
+    *bytes_out = v;
+    return GTR_OK;
+}
+
 // family query hooks (each family's TU)
 int gtr_internal_query_xs(gtr_ctx *, const gtr_launch_cfg *, gtr_variant_info *);
 int gtr_internal_query_su3(gtr_ctx *, const gtr_launch_cfg *, gtr_variant_info *);

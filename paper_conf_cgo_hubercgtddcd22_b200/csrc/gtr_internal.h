@@ -13,7 +13,7 @@ struct gtr_ctx {
     int num_sms;
     uint64_t *pool;
     uint64_t pool_bytes;
-    uint32_t *d_err;       // device error word
+    uint32_t *d_err;       // device error word (+8: fallback high-water mark, u64)
     void *d_stage;         // 256 B staging buffer (e2e request / results)
 };
 
@@ -68,6 +68,7 @@ int resolve(gtr_ctx *ctx, const gtr_launch_cfg *cfg, const void *fn, uint32_t de
     if (per_sm < 1) return GTR_EINVAL;
     L->teams = cfg->num_teams > 0 ? cfg->num_teams : per_sm * ctx->num_sms;
     L->rp.err = ctx->d_err;
+    L->rp.hwm = reinterpret_cast<unsigned long long *>(reinterpret_cast<char *>(ctx->d_err) + 8);
     L->rp.pool = ctx->pool;
     uint64_t hw = (uint64_t)L->teams * (uint64_t)K::BLOCK;
     L->rp.pool_wpt = ctx->pool ? (ctx->pool_bytes / 8u) / hw : 0;

@@ -66,6 +66,7 @@ struct Cfg {
 // Launch-time runtime parameters (host-filled, by value).
 struct RtParams {
     uint32_t *err;              // device error word (ctx-owned)
+    unsigned long long *hwm;    // fallback high-water mark, bytes per thread (ctx-owned)
     uint64_t *pool;             // global fallback pool (caller-owned), may be null
     uint64_t pool_wpt;          // fallback capacity per hardware thread, 8-byte words
     uint32_t sm_stack_words;    // shared-memory stack capacity per thread (words)
@@ -85,6 +86,7 @@ struct TeamState {
     volatile int32_t nvar;      // nthreads-var ICV (omp_set_num_threads)
     uint32_t sb_count;          // software barrier of a partial-warp team:
     volatile uint32_t sb_gen;   //   arrivals and generation
+    volatile uint32_t hwm_seen; // largest fallback bytes/thread this team already reported
     RtParams rp;
     uint64_t bcast[2];          // guarded-value broadcast slots
 };
@@ -278,6 +280,7 @@ template <class K> __device__ __forceinline__ Role team_init(const RtParams &rp)
             g_ts.nvar = K::NT;
             g_ts.sb_count = 0;
             g_ts.sb_gen = 0;
+            g_ts.hwm_seen = 0;
             g_ts.rp = rp;
             return Role::Main;
         }
@@ -290,6 +293,7 @@ template <class K> __device__ __forceinline__ Role team_init(const RtParams &rp)
             g_ts.nvar = K::NT;
             g_ts.sb_count = 0;
             g_ts.sb_gen = 0;
+            g_ts.hwm_seen = 0;
             g_ts.rp = rp;
         }
         __syncthreads();
@@ -436,6 +440,15 @@ template <class K> __device__ __forceinline__ void set_num_threads(int n) {
 // shared memory; when full, the thread's slab of the global fallback pool; when
 // that is exhausted, ERR_HEAP and a per-CTA sink (results declared invalid).
 __device__ __align__(16) static uint64_t g_sink_dummy;
+// Fallback high-water mark: the global atomic only when this team has not
+// yet reported that many bytes (a racy but monotone filter: a few atomics
+// per team instead of one per allocation).
+__device__ __forceinline__ void note_fallback(const RtParams &rp, uint32_t bytes) {
+    if (bytes > g_ts.hwm_seen) {
+        g_ts.hwm_seen = bytes;
+        atomicMax(rp.hwm, (unsigned long long)bytes);
+    }
+}
 template <class K> __device__ __noinline__ void *alloc_shared(uint32_t bytes) {
     const uint32_t words = (bytes + 7u) >> 3;
     ThreadState &ts = tstate<K>();
@@ -450,6 +463,7 @@ template <class K> __device__ __noinline__ void *alloc_shared(uint32_t bytes) {
     if (rp.pool != nullptr && (uint64_t)ts.gsp + words <= rp.pool_wpt) {
         uint64_t *p = rp.pool + ((uint64_t)blockIdx.x * K::BLOCK + threadIdx.x) * rp.pool_wpt + ts.gsp;
         ts.gsp += words;
+        note_fallback(rp, ts.gsp * 8u);          // fallback bytes in use
         return p;
     }
     atomicOr(rp.err, (uint32_t)ERR_HEAP);
@@ -491,6 +505,7 @@ template <class K> __device__ __noinline__ void *alloc_coalesced(uint32_t words,
             uint64_t *p = rp.pool + (uint64_t)gridDim.x * K::BLOCK * half +
                           ((uint64_t)blockIdx.x * K::BLOCK + threadIdx.x) * half + ts.igsp;
             ts.igsp += words;
+            note_fallback(rp, ts.igsp * 8u);
             return p;
         }
         atomicOr(rp.err, (uint32_t)ERR_HEAP);
@@ -512,6 +527,7 @@ template <class K> __device__ __noinline__ void *alloc_coalesced(uint32_t words,
         } else if (rp.pool != nullptr && (uint64_t)W[0].wgtop + words <= 32u * half) {
             p = rp.pool + ((uint64_t)blockIdx.x * K::BLOCK + wbase) * half + W[0].wgtop;
             W[0].wgtop += words;
+            note_fallback(rp, W[0].wgtop * 8u / 32u);   // warp SoA: per lane
             glob = 0x8000u;
         } else {
             k = -1;

@@ -91,6 +91,7 @@ _proto = {
     "gtr_ctx_create": (_i, [_i, _vp, _u64, _P(_vp)]),
     "gtr_ctx_destroy": (_i, [_vp]),
     "gtr_ctx_check": (_i, [_vp, _vp]),
+    "gtr_ctx_fallback_high_water": (_i, [_vp, C.POINTER(C.c_uint64), C.c_int32, _vp]),
     "gtr_query_variant": (_i, [_i, _P(gtr_launch_cfg), _P(gtr_variant_info)]),
     "gtr_forkjoin": (_i, [_vp, _P(gtr_launch_cfg), _i64, C.c_int32, C.c_int32, _vp, _vp]),
     "gtr_barrier_floor": (_i, [_vp, _P(gtr_launch_cfg), _i64, _vp, _vp]),
@@ -168,6 +169,15 @@ def gtr_ctx_destroy(ctx):
 def gtr_ctx_check(ctx, stream=None, raise_on_error=True):
     st = _lib.gtr_ctx_check(ctx, _stream(stream))
     return _check("gtr_ctx_check", st) if raise_on_error else st
+
+
+def gtr_ctx_fallback_high_water(ctx, reset=False, stream=None):
+    """Largest bytes of globalized variables one thread held in the global
+    fallback pool since creation / the last reset."""
+    v = C.c_uint64(0)
+    _check("gtr_ctx_fallback_high_water", _lib.gtr_ctx_fallback_high_water(ctx, C.byref(v), 1 if reset else 0,
+                                                                            _stream(stream)))
+    return int(v.value)
 
 
 def gtr_query_variant(kernel, launch_cfg):

@@ -162,6 +162,28 @@ def test_runtime_stack_overflow_falls_back_to_pool(G, ctx, dev_small, small):
         _assert_same(out, v, o_out, o_v)
 
 
+def test_fallback_high_water_mark(G, ctx, dev_small, small):
+    """gtr_ctx_fallback_high_water: 0 when every globalized variable stays in
+    registers / shared memory; with the forced global placement the lookup's
+    locals (seed 8 B, macro_xs 40 B, xs 40 B, AMB-7) live in the pool -- at
+    least the accumulation region's 80 B at once, and never more than the
+    88 B of all three plus the main thread's 16-byte chunk struct."""
+    t, P, o_out, o_v, n = small
+    G.gtr_ctx_fallback_high_water(ctx, reset=True)
+    for m in (G.SPMD, G.CSM):
+        _run(G, ctx, dev_small, G.cfg(m, G.PL_STACK, 1, 128), 0, 20000, verify=False)
+    assert G.gtr_ctx_fallback_high_water(ctx, reset=True) == 0
+    for m in (G.SPMD, G.GENERIC):
+        _run(G, ctx, dev_small, G.cfg(m, G.PL_GLOBAL, 0, 128), 0, 20000, verify=False)
+        hw = G.gtr_ctx_fallback_high_water(ctx, reset=True)
+        assert 80 <= hw <= 104 and hw % 8 == 0, (m, hw)
+    # the runtime placement spills past a 16-byte shared stack into the pool
+    _run(G, ctx, dev_small, G.cfg(G.SPMD, G.PL_RUNTIME, 0, 128, smem_stack_bytes=16), 0, 20000, verify=False)
+    assert G.gtr_ctx_fallback_high_water(ctx, reset=True) > 0
+    _run(G, ctx, dev_small, G.cfg(G.SPMD, G.PL_RUNTIME, 0, 128), 0, 20000, verify=False)
+    assert G.gtr_ctx_fallback_high_water(ctx) == 0
+
+
 def test_heap_exhaustion_reports_eheap(G, dev_small):
     # no fallback pool at all: GTR_PL_GLOBAL cannot allocate -> GTR_EHEAP
     c = G.gtr_ctx_create(0, None, 0)
