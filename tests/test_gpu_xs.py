@@ -95,6 +95,26 @@ def test_energies_outside_the_grid(G, ctx, orc, log2b):
         _assert_same(out, v, o_out, o_v)
 
 
+def test_energy_exactly_one(G, ctx, dev_small, dev_small_plain, small):
+    """A lookup seed whose first draw is 2^63 - 1: u64 -> f64 rounds it to
+    2^63, so E = 1.0 exactly (c1.1) -- the top edge of the last union bin.
+    Lookups 0..63 of that seed through both search paths vs the oracle."""
+    t, P, *_ = small
+    a, M = 2806196910506780709, 1 << 63
+    a_inv = pow(a, -1, M)
+    seed = (a_inv * ((M - 1) - 1)) % M            # a * seed + 1 = 2^63 - 1
+    o_out, o_v = P.run(0, 64, seed, 1, verify=True)
+    assert o_v["u"][0] == P.n_union - 2          # E = 1.0 is above every energy
+    for dev in (dev_small, dev_small_plain):
+        for c in (G.cfg(G.SPMD, G.PL_STACK, 1, 256), G.cfg(G.NATIVE, G.PL_STACK, 1, 256),
+                  G.cfg(G.CSM, G.PL_STACK, 1, 128, flags=G.F_PLAIN)):
+            out = torch.zeros(18, dtype=torch.uint64, device="cuda")
+            v, bufs = dev.verify_buffers(64)
+            G.gtr_xs_lookup(ctx, c, dev.tables, 0, 64, seed, out, v)
+            G.gtr_ctx_check(ctx)
+            _assert_same(out.cpu().numpy(), {k: b.cpu().numpy() for k, b in bufs.items()}, o_out, o_v)
+
+
 def _run(G, ctx, dev, cfg, first, n, verify=True):
     out = torch.zeros(18, dtype=torch.uint64, device="cuda")
     v, bufs = dev.verify_buffers(n) if verify else (None, None)
