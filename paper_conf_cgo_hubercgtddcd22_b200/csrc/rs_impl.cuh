@@ -56,6 +56,9 @@ __device__ __forceinline__ double cabs_(cx a) { return sqrt(a.r * a.r + a.i * a.
 #ifndef GTR_RS_PREFETCH
 #define GTR_RS_PREFETCH 1
 #endif
+#ifndef GTR_RS_PCOPY
+#define GTR_RS_PCOPY 0   // measured: the copy spills at 128 registers, 104.1 -> 99.8 M lookups/s
+#endif
 __device__ __forceinline__ void ld256(const double *a, double &x0, double &x1, double &x2, double &x3) {
     asm("ld.global.nc.v4.f64 {%0, %1, %2, %3}, [%4];" : "=d"(x0), "=d"(x1), "=d"(x2), "=d"(x3) : "l"(a));
 }
@@ -355,8 +358,13 @@ template <class K> struct BucketRegion {
         const Chunk *c = static_cast<const Chunk *>(a);
         const uint64_t base = c->base, cnt = c->count;
         ChunkBuf<K> &b = chunk_buf<K>();
+#if GTR_RS_PCOPY
+        const Params P = g_p;      // register copy (g_p is shared memory; see xs_impl.cuh)
+#else
+        const Params &P = g_p;
+#endif
         for_dynamic_warp<K>(0, (int64_t)cnt, &b.next,
-                            [&](int64_t q) { lookup<K>(g_p, base + b.perm[q], g_tally); });
+                            [&](int64_t q) { lookup<K>(P, base + b.perm[q], g_tally); });
     }
 };
 
