@@ -46,3 +46,14 @@ def test_oracle_is_not_reachable_from_product():
                 txt = open(os.path.join(dp, f)).read()
                 assert "import oracle" not in txt and "from oracle" not in txt, f
                 assert "oracle.h" not in txt and "liboracle" not in txt, f
+
+
+def test_product_fails_loudly_without_library():
+    """No CPU fallback: with the CUDA library absent the binding refuses to import."""
+    import subprocess
+    import sys
+    env = dict(os.environ, GTR_LIB=os.path.join(ROOT, "build", "does_not_exist", "libgtr.so"))
+    r = subprocess.run([sys.executable, "-c", "import paper_conf_cgo_hubercgtddcd22_b200.gtr"],
+                       cwd=ROOT, env=env, capture_output=True, text=True)
+    assert r.returncode != 0
+    assert "ImportError" in r.stderr and "no CPU fallback" in r.stderr
