@@ -56,6 +56,12 @@ __device__ __forceinline__ double cabs_(cx a) { return sqrt(a.r * a.r + a.i * a.
 #ifndef GTR_RS_PREFETCH
 #define GTR_RS_PREFETCH 1
 #endif
+#ifndef GTR_RS_PRESUF
+#define GTR_RS_PRESUF 0
+#endif
+#ifndef GTR_RS_SF_SELECT
+#define GTR_RS_SF_SELECT 0
+#endif
 #ifndef GTR_RS_PCOPY
 #define GTR_RS_PCOPY 0   // measured: the copy spills at 128 registers, 104.1 -> 99.8 M lookups/s
 #endif
@@ -100,6 +106,35 @@ __device__ __forceinline__ cx faddeeva_series(cx Z) {
         const cx den = {12.0 * Z.r, 12.0 * Z.i};                        // 12 Z
         const double b_r = 144.0 * (Z.r * Z.r - Z.i * Z.i), b_i = 144.0 * (2.0 * Z.r * Z.i);   // 144 Z^2
         // batched inversion of q_0 = |12 Z|^2, q_{n+1} = |dl_n - 144 Z^2|^2
+#if GTR_RS_PRESUF
+        // prefix and suffix products side by side (two independent chains of
+        // 10 instead of prefix -> reciprocal -> backward sweep): 1/q_n =
+        // pre[n] * suf[n+1] / P, a shorter dependent path per pole
+        double q[11], pre[11], suf[12];
+        q[0] = den.r * den.r + den.i * den.i;
+#pragma unroll
+        for (int n = 0; n < 10; n++) {
+            const double br = dl[n] - b_r;
+            q[n + 1] = br * br + b_i * b_i;
+        }
+        pre[0] = 1.0;
+        suf[11] = 1.0;
+#pragma unroll
+        for (int n = 0; n < 10; n++) {
+            pre[n + 1] = pre[n] * q[n];
+            suf[10 - n] = suf[11 - n] * q[10 - n];
+        }
+        const double invP = 1.0 / (pre[10] * q[10]);
+        cx Se = {0.0, 0.0}, So = {0.0, 0.0};
+#pragma unroll
+        for (int n = 9; n >= 0; n--) {
+            const double br = dl[n] - b_r;
+            const double w = an[n] * ((pre[n + 1] * suf[n + 2]) * invP);  // an / q_{n+1}
+            if (n & 1) { So.r += w * br; So.i += w * b_i; }
+            else       { Se.r += w * br; Se.i += w * b_i; }
+        }
+        const double inv = (pre[0] * suf[1]) * invP;                      // 1 / q_0
+#else
         double pre[11];
         pre[0] = den.r * den.r + den.i * den.i;
 #pragma unroll
@@ -117,6 +152,7 @@ __device__ __forceinline__ cx faddeeva_series(cx Z) {
             if (n & 1) { So.r += w * br; So.i += w * b_i; }             // an conj(bot_n) / |bot_n|^2
             else       { Se.r += w * br; Se.i += w * b_i; }
         }
+#endif
         // W0 = i (1 - e) / (12 Z) = {e.i, 1 - e.r} conj(den) / |den|^2
         const double nr = e.i, ni = 1.0 - e.r;
         const cx W0 = {(nr * den.r + ni * den.i) * inv, (ni * den.r - nr * den.i) * inv};
@@ -199,7 +235,17 @@ __device__ __forceinline__ void micro_xs(const Params &P, int64_t nuc, double E,
         Wv[0] = W.r;
         Wv[1] = W.i;
         const cx Wl = {Wv[0], Wv[1]};
+#if GTR_RS_SF_SELECT
+        // constant indices only: in the heap-to-stack placement the factors
+        // stay in registers (a runtime index puts the array in local memory,
+        // one 16-byte LDL per pole)
+        cx f = {sf[0], sf[1]};
+        if (lv == 1) f = cx{sf[2], sf[3]};
+        if (lv == 2) f = cx{sf[4], sf[5]};
+        if (lv == 3) f = cx{sf[6], sf[7]};
+#else
         const cx f = {sf[2 * lv], sf[2 * lv + 1]};
+#endif
         sig[0] = sig[0] + cmul(cx{RT.x, RT.y}, cmul(Wl, f)).r;
         sig[1] = sig[1] + cmul(cx{RA.x, RA.y}, Wl).r;
         sig[2] = sig[2] + cmul(cx{RF.x, RF.y}, Wl).r;
