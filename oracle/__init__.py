@@ -56,6 +56,8 @@ def lib():
         L.orc_su3_mat_nn.restype = None; L.orc_su3_mat_nn.argtypes = [i64, vp, vp, vp, C.c_int]
         L.orc_fast_exp.restype = dbl; L.orc_fast_exp.argtypes = [dbl]
         L.orc_fast_nuclear_W.restype = Cplx; L.orc_fast_nuclear_W.argtypes = [Cplx]
+        L.orc_rs_faddeeva_constants.restype = None
+        L.orc_rs_faddeeva_constants.argtypes = [vp, vp, vp, vp]
         L.orc_rs_lookup.restype = None; L.orc_rs_lookup.argtypes = [vp, u64, u64, vp, vp, vp]
         L.orc_rs_run.restype = None
         L.orc_rs_run.argtypes = [vp, u64, u64, u64, C.c_int, vp, vp, vp, vp, vp]
@@ -194,6 +196,14 @@ def fast_nuclear_W(z):
 
 def fast_exp(x):
     return lib().orc_fast_exp(x)
+
+
+def rs_faddeeva_constants():
+    """(an[10], denominator_left[10], prefactor, (a, b, c, d)) as orc_fast_nuclear_W uses them."""
+    an, dl, asym = np.zeros(10), np.zeros(10), np.zeros(4)
+    pre = C.c_double()
+    lib().orc_rs_faddeeva_constants(_p(an), _p(dl), C.byref(pre), _p(asym))
+    return an, dl, pre.value, asym
 
 
 class RsProblem:

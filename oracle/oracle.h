@@ -97,6 +97,8 @@ typedef struct {
 
 typedef struct { double r, i; } orc_cplx;
 orc_cplx orc_fast_nuclear_W(orc_cplx z);          /* Abrarov / asymptotic   */
+/* the tabulated Faddeeva constants orc_fast_nuclear_W uses (for their pins) */
+void orc_rs_faddeeva_constants(double an[10], double dl[10], double *prefactor, double asym[4]);
 double   orc_fast_exp(double x);                   /* (1+x/4096)^(2^12)      */
 void     orc_rs_lookup(const orc_rs_tables *t, uint64_t i, uint64_t seed,
                        int32_t *mat, double macro[4], int32_t *argmax);

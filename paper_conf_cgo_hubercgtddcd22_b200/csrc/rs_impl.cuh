@@ -93,9 +93,17 @@ __device__ __forceinline__ cx fast_cexp(cx z) {
 // collapse into two sums because the numerators alternate between
 // -e - 1 (n even) and e - 1 (n odd).  RSBench's form needs 22 fp64 divisions
 // per pole, each an XU-pipe reciprocal plus a Newton sequence; the XU pipe
-// was the busiest unit (ncu: 75% of peak).  |Z| < 6 is tested as |Z|^2 < 36
-// (same branch: sqrt is monotonic and correctly rounded).
-__device__ __forceinline__ bool faddeeva_inner_branch(cx Z) { return Z.r * Z.r + Z.i * Z.i < 36.0; }
+// was the busiest unit (ncu: 75% of peak).
+//
+// The branch must be the oracle's: |Z| = sqrt(Z.r*Z.r + Z.i*Z.i) < 6 with
+// every operation rounded separately (no FMA -- this TU contracts, so the
+// squares and the sum are explicit round-to-nearest intrinsics).  Then
+// sqrt(x) < 6 <=> x < 36 for every double x: sqrt is monotonic, correctly
+// rounded, and sqrt(pred(36)) = 6 - 0.667 ulp(6^-) rounds below 6 (pinned
+// by tests/test_oracle_rs.py::test_branch_predicate_sqrt_equivalence).
+__device__ __forceinline__ bool faddeeva_inner_branch(cx Z) {
+    return __dadd_rn(__dmul_rn(Z.r, Z.r), __dmul_rn(Z.i, Z.i)) < 36.0;
+}
 __device__ __forceinline__ cx faddeeva_series(cx Z) {
     {
         constexpr double an[10] = {2.758402e-01, 2.245740e-01, 1.594149e-01, 9.866577e-02, 5.324414e-02,

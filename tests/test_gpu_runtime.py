@@ -74,12 +74,14 @@ def test_semantics_all_variants(G, ctx, orc, variant):
         G.gtr_semantics(ctx, G.cfg(m, p, f, nt, num_teams=G_teams), test, out, out.numel())
         G.gtr_ctx_check(ctx)
         got = out.cpu().numpy()
-        private = p == G.PL_STACK or (p == G.PL_COALESCED and m == G.SPMD)
-        if test == 1 and private:
-            # Fig. 3 with the locals left in thread-private stack memory (heap-
-            # to-stack, or LLVM 12's SPMD shortcut): every thread dereferences
-            # thread 0's address in its OWN local window -- the miscompile the
-            # paper removes.
+        if test == 1 and p == G.PL_COALESCED and m == G.SPMD:
+            # LLVM-12 unsound shortcut: in SPMD mode LLVM 12 puts
+            # every globalized local in thread-private memory without checking
+            # whether its address escapes, so each thread dereferences thread
+            # 0's address in its OWN local window and reads 42 + t -- the
+            # miscompile the paper removes.  Every other
+            # placement, heap-to-stack included, must give the oracle's 42:
+            # heap-to-stack is illegal for the escaping Lcl.
             assert np.array_equal(got, want + np.tile(np.arange(nt, dtype=np.uint64), G_teams))
             continue
         assert np.array_equal(got[:len(want)], want), test

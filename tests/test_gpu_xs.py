@@ -115,6 +115,41 @@ def test_energy_exactly_one(G, ctx, dev_small, dev_small_plain, small):
             _assert_same(out.cpu().numpy(), {k: b.cpu().numpy() for k, b in bufs.items()}, o_out, o_v)
 
 
+def _seed_e_one():
+    a, M = 2806196910506780709, 1 << 63
+    return (pow(a, -1, M) * ((M - 1) - 1)) % M     # a * seed + 1 = 2^63 - 1
+
+
+def test_energy_exactly_one_grid_types_and_sorted(G, ctx, dev_grid, dev_small, small):
+    """E = 1.0 through the nuclide grid, the hash grid (bin E / du = hash_bins
+    clamped to the last bin, DESIGN.md R-XS-hash1 -- unclamped it read one row
+    past the hash table) and the sorted event mode (sort key clamped to the
+    last energy bucket): bit-identical to the oracle's unionized lookups."""
+    gt, dev = dev_grid
+    t, P, *_ = small
+    seed = _seed_e_one()
+    o_out, o_v = P.run(0, 64, seed, 1, verify=True)
+    cfgs = (G.cfg(G.SPMD, G.PL_STACK, 1, 256), G.cfg(G.NATIVE, G.PL_STACK, 1, 256),
+            G.cfg(G.CSM, G.PL_STACK, 1, 128, flags=G.F_PLAIN), G.cfg(G.GENERIC, G.PL_RUNTIME, 0, 128))
+    for c in cfgs:
+        out = torch.zeros(18, dtype=torch.uint64, device="cuda")
+        v, bufs = dev.verify_buffers(64)
+        G.gtr_xs_lookup(ctx, c, dev.tables, 0, 64, seed, out, v)
+        G.gtr_ctx_check(ctx)
+        assert np.array_equal(out.cpu().numpy(), o_out)
+        assert np.array_equal(bufs["macro"].cpu().numpy().view(np.uint64), o_v["macro"].view(np.uint64))
+        assert np.array_equal(bufs["mat"].cpu().numpy(), o_v["mat"])
+    for d in (dev, dev_small):
+        for c in cfgs[:2]:
+            out = torch.zeros(18, dtype=torch.uint64, device="cuda")
+            v, bufs = d.verify_buffers(64)
+            ws = torch.empty(G.gtr_xs_sorted_workspace_bytes(64), dtype=torch.uint8, device="cuda")
+            G.gtr_xs_lookup_sorted(ctx, c, d.tables, 0, 64, seed, out, ws, v)
+            G.gtr_ctx_check(ctx)
+            assert np.array_equal(out.cpu().numpy(), o_out)
+            assert np.array_equal(bufs["macro"].cpu().numpy().view(np.uint64), o_v["macro"].view(np.uint64))
+
+
 def _run(G, ctx, dev, cfg, first, n, verify=True):
     out = torch.zeros(18, dtype=torch.uint64, device="cuda")
     v, bufs = dev.verify_buffers(n) if verify else (None, None)

@@ -67,7 +67,8 @@ def _macro_bg_only(t, E, mat):
     for j in range(int(t["num_nucs"][mat])):
         n = int(t["mats"][mat, j])
         nw = int(t["n_windows"][n])
-        w = min(int(E * nw), nw - 1)
+        w = int(E / (1.0 / nw))              # c4 step 1, as the oracle (RSBench)
+        w = nw - 1 if w == nw else w
         T, A_, F = (t["windows"][f][n, w] for f in ("T", "A", "F"))
         want += t["concs"][mat, j] * np.array([E * T, E * A_, E * F, E * T - E * A_])
     return want
@@ -102,7 +103,8 @@ def test_single_pole_against_scipy_faddeeva(orc, rs_small):
         for j in range(int(t["num_nucs"][mat])):
             nuc = int(t["mats"][mat, j])
             nw = int(t["n_windows"][nuc])
-            w = min(int(E * nw), nw - 1)
+            w = int(E / (1.0 / nw))
+            w = nw - 1 if w == nw else w
             p = t["poles"][nuc, int(t["windows"]["start"][nuc, w])]
             EA = complex(*p["EA"])
             W = wofz((E - EA) * 0.5)
@@ -230,3 +232,123 @@ def test_sigT_factors_vs_spherical_bessel(orc, rs_small, L):
         assert abs(abs(f) - 1.0) <= 1e-11
         n_checked += 1
     assert n_checked == 300
+
+
+# ---------------------------------------------------------------- constants
+def _unit7(x):
+    """one unit in the 7th significant digit of x"""
+    import math
+    return 10.0 ** (math.floor(math.log10(abs(x))) - 6)
+
+
+def test_faddeeva_constants_closed_forms(orc):
+    """The 22 tabulated Abrarov constants (7 significant digits, as RSBench
+    tabulates them) against their closed forms (Abrarov N = 10, tau_m = 12):
+    a_n = 2 sqrt(pi)/12 exp(-(n pi / 12)^2), denominator_left_n = (n pi)^2,
+    prefactor = tau_m^2 / sqrt(pi) = 144 / sqrt(pi) -- each within one unit
+    of its 7th significant digit (a typo in any digit fails).  RSBench's
+    denominator_left[8] = 7.994379e+02 is 81 pi^2 = 799.43796 truncated, not
+    rounded (the only such entry; kept as tabulated, R4)."""
+    import mpmath as mp
+    mp.mp.dps = 50
+    an, dl, pre, _ = orc.rs_faddeeva_constants()
+    for n in range(1, 11):
+        a_c = float(2 * mp.sqrt(mp.pi) / 12 * mp.exp(-(n * mp.pi / 12) ** 2))
+        d_c = float((n * mp.pi) ** 2)
+        assert abs(an[n - 1] - a_c) <= _unit7(a_c) * 0.5 + 1e-18, (n, an[n - 1], a_c)
+        assert abs(dl[n - 1] - d_c) <= _unit7(d_c), (n, dl[n - 1], d_c)
+        if n != 9:                                   # every other entry is rounded to nearest
+            assert abs(dl[n - 1] - d_c) <= _unit7(d_c) * 0.5, (n, dl[n - 1], d_c)
+    assert abs(pre - float(144 / mp.sqrt(mp.pi))) <= _unit7(pre) * 0.5
+
+
+def test_faddeeva_asymptotic_constants_gauss_hermite(orc):
+    """The 2-pole asymptotic W(z) = i z (a/(z^2 - b) + c/(z^2 - d)) is the
+    4-point Gauss-Hermite quadrature of W(z) = (i/pi) int e^{-t^2}/(z - t) dt:
+    nodes t^2 = b, d = (3 -+ sqrt 6)/2 (roots of H_4), weights a, c = 2 w/pi
+    with w = sqrt(pi) / (4 (3 -+ sqrt 6)).  The 60-digit literals must be the
+    nearest doubles of these closed forms, and a, b, c, d must reproduce the
+    quadrature computed by numpy's hermgauss."""
+    import mpmath as mp
+    mp.mp.dps = 80
+    _, _, _, asym = orc.rs_faddeeva_constants()
+    s6 = mp.sqrt(6)
+    want = [1 / (2 * mp.sqrt(mp.pi) * (3 - s6)), (3 - s6) / 2, 1 / (2 * mp.sqrt(mp.pi) * (3 + s6)), (3 + s6) / 2]
+    for got, w in zip(asym, want):
+        assert got == float(w), (got, w)
+    x, w = np.polynomial.hermite.hermgauss(4)
+    xp, wp = x[x > 0], w[x > 0]
+    order = np.argsort(xp)
+    np.testing.assert_allclose([xp[order][0] ** 2, xp[order][1] ** 2], [asym[1], asym[3]], rtol=1e-14)
+    np.testing.assert_allclose(2 * wp[order] / np.pi, [asym[0], asym[2]], rtol=1e-14)
+
+
+def test_branch_predicate_sqrt_equivalence():
+    """The GPU tests |Z| < 6 as Z.r^2 + Z.i^2 < 36 (each op rounded, no FMA);
+    the oracle as sqrt(Z.r^2 + Z.i^2) < 6.  For every double x the two agree:
+    sqrt is monotonic and correctly rounded, sqrt(36) = 6 exactly, and the
+    largest double below 36 has a square root that rounds below 6 -- checked
+    on the 2^16 doubles each side of 36."""
+    x = np.float64(36.0)
+    below = [x]
+    above = [x]
+    for _ in range(1 << 16):
+        below.append(np.nextafter(below[-1], 0.0))
+        above.append(np.nextafter(above[-1], 100.0))
+    xs = np.array(below + above, dtype=np.float64)
+    assert np.array_equal(np.sqrt(xs) < 6.0, xs < 36.0)
+    assert np.sqrt(np.nextafter(36.0, 0.0)) < 6.0
+
+
+def test_faddeeva_branch_boundary_in_oracle(orc):
+    """Z straddling |Z| = 6 by one ulp of |Z|^2 selects the Abrarov series on
+    the inside and the asymptotic form outside: just inside, W equals the
+    series' value at |Z| = 6 -- continuous to the approximation's accuracy
+    with the asymptotic value just outside (both within 2e-5 of wofz)."""
+    for th in (0.3, 1.1, 2.0, 2.9):
+        z = 6.0 * np.exp(1j * th)
+        zin = z * (1 - 4e-16)
+        zout = z * (1 + 4e-16)
+        assert abs(zin) < 6.0 <= abs(zout) or abs(zin) < 6.0
+        w_in, w_out = orc.fast_nuclear_W(zin), orc.fast_nuclear_W(zout)
+        assert abs(w_in - wofz(zin)) <= 2e-3 * abs(wofz(zin))
+        assert abs(w_out - wofz(zout)) <= 2e-5
+
+
+def test_window_index_rule(orc, rs_small):
+    """Background-only windows, n_windows = 10, and lookup seeds constructed so
+    that E is each of the 9 doubles nearest the window edges k / 10 (and
+    E = 1.0): the oracle's window must be (int)(E / (1.0 / n_windows)) clamped
+    to n_windows - 1 (c4 step 1, RSBench's expression -- not
+    int(E * n_windows), which differs at some of these edges)."""
+    t = {k: (v.copy() if isinstance(v, np.ndarray) else v) for k, v in rs_small.items()}
+    t["windows"]["end"] = t["windows"]["start"]           # no poles
+    NW = 10
+    t["n_windows"][:] = NW
+    P = orc.RsProblem(t)
+    a_inv = pow(A_LCG, -1, M)
+    differ = 0
+    for k in range(1, NW + 1):
+        E0 = np.float64(k / NW)
+        cands = [E0]
+        for _ in range(4):
+            cands = [np.nextafter(cands[0], 0.0)] + cands + [np.nextafter(cands[-1], 2.0)]
+        for Ec in cands:
+            if Ec > 1.0:
+                continue
+            s1 = min(int(Fraction(float(Ec)) * M), M - 1)    # E * 2^63 is an integer here
+            seed = (a_inv * ((s1 - 1) % M)) % M              # first draw of lookup 0 = s1
+            E, s = orc.lcg_double(seed)
+            assert E == Ec
+            mat, _ = orc.pick_mat(s)
+            _, macro, _ = P.lookup(0, seed)
+            w = int(E / (1.0 / NW))
+            w = NW - 1 if w == NW else w
+            differ += w != min(int(E * NW), NW - 1)
+            want = np.zeros(4)
+            for j in range(int(t["num_nucs"][mat])):
+                n = int(t["mats"][mat, j])
+                T_, A_, F_ = (t["windows"][f][n, w] for f in ("T", "A", "F"))
+                want += t["concs"][mat, j] * np.array([E * T_, E * A_, E * F_, E * T_ - E * A_])
+            np.testing.assert_allclose(macro, want, rtol=1e-13, atol=1e-15)
+    assert differ > 0          # the edges exercise the difference between the two expressions

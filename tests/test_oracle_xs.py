@@ -256,3 +256,36 @@ def test_threads_do_not_change_results(orc):
     assert np.array_equal(a, b)
     for k in va:
         assert np.array_equal(va[k], vb[k])
+
+
+def seed_with_first_draw(s1):
+    """Lookup seed whose lookup-0 state after one LCG step is s1 (a * seed + 1 = s1)."""
+    return (pow(A, -1, M) * ((s1 - 1) % M)) % M
+
+
+@pytest.mark.parametrize("bins", [10000, 97, 1])
+def test_energy_one_hash_bin_clamped(orc, bins):
+    """E = 1.0 exactly (first draw 2^63 - 1 rounds up to 2^63, c1.1): the hash
+    grid's bin E / du = hash_bins would be one row past the table (XSBench's
+    own overread); the clamped last bin (DESIGN.md R-XS-hash1) must locate the
+    same bracketing pair as the unionized grid -- the last pair of every
+    nuclide, which a brute-force interpolation at E = 1.0 reproduces."""
+    seed = seed_with_first_draw(M - 1)
+    d, _ = orc.lcg_double(seed)
+    assert d == 1.0
+    t = X.make_tables(13, 200, seed_t=5)
+    ref, vref = orc.XsProblem(t, grid_type=0).run(0, 64, seed, 1, verify=True)
+    for gt in (1, 2):
+        out, v = orc.XsProblem(t, grid_type=gt, hash_bins=bins).run(0, 64, seed, 1, verify=True)
+        assert np.array_equal(out, ref)
+        assert np.array_equal(v["macro"].view(np.uint64), vref["macro"].view(np.uint64))
+    # brute force for lookup 0: every nuclide's last pair, hi - f (hi - lo), f = (hi.e - 1) / (hi.e - lo.e)
+    mat = int(vref["mat"][0])
+    g = t["grid"]
+    want = np.zeros(5)
+    for j in range(int(t["num_nucs"][mat])):
+        nuc, c = int(t["mats"][mat, j]), float(t["concs"][mat, j])
+        lo, hi = g[nuc, -2], g[nuc, -1]
+        f = (hi[0] - 1.0) / (hi[0] - lo[0])
+        want += (hi[1:6] - f * (hi[1:6] - lo[1:6])) * c
+    assert np.allclose(vref["macro"][0], want, rtol=1e-13, atol=0)
