@@ -6,13 +6,15 @@ indirect call may reach every address-taken function of the module (the
 registers and even their static shared memory.  Each application in the paper
 is its own module, so each GENERIC/CASCADE variant is compiled as its own
 translation unit here; CSM and SPMD variants (no function pointers) are
-grouped per thread_limit.  Objects are cached under build/ by flags+mtime.
+grouped per thread_limit.  Objects are cached under build/ by flags + the mtime of the source and
+the headers it includes.
 
     python -m paper_conf_cgo_hubercgtddcd22_b200.build [-j N] [--force]
 """
 import argparse
 import hashlib
 import os
+import re
 import shutil
 import subprocess
 import sys
@@ -60,17 +62,26 @@ def units():
     return out
 
 
-def _deps_mtime():
-    m = 0.0
-    for d in (CSRC, os.path.join(ROOT, "include")):
-        for f in os.listdir(d):
-            if f.endswith((".cu", ".cuh", ".h")):
-                m = max(m, os.path.getmtime(os.path.join(d, f)))
+_INC = re.compile(r'^\s*#\s*include\s+"([^"]+)"', re.M)
+
+
+def _deps_mtime(src, seen=None):
+    """Newest mtime of `src` and every file it #includes with quotes (recursively)."""
+    seen = set() if seen is None else seen
+    path = os.path.normpath(src if os.path.isabs(src) else os.path.join(CSRC, src))
+    if path in seen or not os.path.exists(path):
+        return 0.0
+    seen.add(path)
+    m = os.path.getmtime(path)
+    with open(path) as f:
+        for inc in _INC.findall(f.read()):
+            m = max(m, _deps_mtime(os.path.join(os.path.dirname(path), inc), seen))
     return m
 
 
-def _compile(job, force, deps_m):
+def _compile(job, force):
     name, src, defs = job
+    deps_m = _deps_mtime(src)
     flags = CFLAGS + defs
     if src.startswith("rs"):
         # RS parity is within a tolerance (libm sin/cos/atan differ anyway,
@@ -91,11 +102,10 @@ def _compile(job, force, deps_m):
 
 def build(jobs=None, force=False, verbose=True):
     os.makedirs(OBJ, exist_ok=True)
-    deps_m = _deps_mtime()
     us = units()
     jobs = jobs or max(1, os.cpu_count() or 1)
     with ThreadPoolExecutor(jobs) as ex:
-        res = list(ex.map(lambda j: _compile(j, force, deps_m), us))
+        res = list(ex.map(lambda j: _compile(j, force), us))
     errs = [e for _, e in res if e]
     if errs:
         raise RuntimeError("nvcc failed:\n" + "\n".join(errs[:3]))
