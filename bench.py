@@ -43,6 +43,9 @@ def parse():
     ap.add_argument("--impl", default="gtr", choices=["gtr", "reference"])
     ap.add_argument("--no-sweep", action="store_true", help="skip the per-mode / fork-join sweeps")
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--combine", default="auto", choices=["auto", "fused", "nccl"],
+                    help="N > 1: combine of the 18 u64 results -- fused into the lookup kernel's epilogue over "
+                         "peer memory (auto: if every rank set it up and it matches NCCL once), or NCCL all_reduce")
     return ap.parse_args()
 
 
@@ -127,6 +130,105 @@ def cpu_baseline(tables, first, n, seed):
             "seconds": dt}, out
 
 
+def host_info():
+    """nproc and the CPU model (lscpu) of the box the oracle baselines ran on."""
+    model = None
+    try:
+        out = subprocess.run(["lscpu"], capture_output=True, text=True, timeout=10).stdout
+        for l in out.splitlines():
+            if l.startswith("Model name:"):
+                model = l.split(":", 1)[1].strip()
+    except (OSError, subprocess.TimeoutExpired):
+        pass
+    if model is None and os.path.exists("/proc/cpuinfo"):
+        for l in open("/proc/cpuinfo"):
+            if l.startswith("model name"):
+                model = l.split(":", 1)[1].strip()
+                break
+    return {"nproc": os.cpu_count(), "cpu_model": model}
+
+
+def oracle_fj(nt, R=20000):
+    """Config 2 beside the GPU: the oracle's host team (main + min(thread_limit,
+    nproc) pthreads, pthread_barrier fork and join), ns per fork/join."""
+    import oracle
+    T = max(1, min(nt, os.cpu_count() or 1))
+    res = {"threads": T, "regions": R}
+    for tag, body, K in (("empty", 0, 1), ("trivial_k4", 1, 4)):
+        r, ns = oracle.fj_host_team(T, R, body, K)
+        assert r == oracle.fj_team(0, T, R, body, K)
+        res[f"{tag}_ns"] = ns
+    return res
+
+
+def oracle_su3(sites=32 ** 4, reps=3):
+    """Config 3 beside the GPU: the oracle on nproc threads over the 32^4
+    lattice (constant inputs), best of `reps`, ms per iteration."""
+    import gtr_inputs.su3 as S
+    import oracle
+    A, B = S.make_lattice(sites, "constant")
+    cores = os.cpu_count() or 1
+    best = None
+    for _ in range(reps):
+        t0 = time.perf_counter()
+        Cm = oracle.su3_mat_nn(A, B, cores)
+        dt = time.perf_counter() - t0
+        best = dt if best is None else min(best, dt)
+    ok = bool(np.all(Cm.real == 1.0) and np.all(Cm.imag == 0.0))
+    return {"ms_per_iter": best * 1e3, "gb_s": sites * 1152 / best / 1e9, "cores": cores, "kind": "oracle",
+            "closed_form_ok": ok, "sample": f"full 32^4 lattice, {cores} pthreads, best of {reps}"}
+
+
+def oracle_rs(n=100_000):
+    """Config 4 beside the GPU: the oracle on nproc threads over a bounded
+    sample of the 10M-lookup workload (lookups [0, n)), lookups/s."""
+    import gtr_inputs.rs as RS
+    import gtr_inputs.xs as X
+    import oracle
+    P = oracle.RsProblem(RS.make_tables())
+    cores = os.cpu_count() or 1
+    t0 = time.perf_counter()
+    out, _, _ = P.run(0, n, X.SEED_L, cores)
+    dt = time.perf_counter() - t0
+    return {"lookups_per_s": n / dt, "cores": cores, "kind": "oracle",
+            "sample": f"lookups [0, {n}) of the 10M workload, {cores} pthreads, table build excluded"}, out
+
+
+def xs_small_config(G, torch, ctx, stream):
+    """Config 1 (XS small: 68 nuclides x 11,303, 1e5 lookups): the GPU's SPMD
+    and NATIVE lookups/s beside the oracle's full run on 1 core and on nproc
+    threads (table build excluded), results compared."""
+    import gtr_inputs.xs as X
+    import oracle
+    from paper_conf_cgo_hubercgtddcd22_b200.problems import XsDevice
+    t = X.make_tables(68, N_GP)
+    n = 100_000
+    xs = XsDevice(ctx, t)
+    out = torch.zeros(18, dtype=torch.uint64, device="cuda")
+    res = {"workload": "XSBench small: 68 nuclides x 11,303 gridpoints, 100,000 lookups"}
+    P = oracle.XsProblem(t)
+    cores = os.cpu_count() or 1
+    t0 = time.perf_counter()
+    o1, _ = P.run(0, n, X.SEED_L, 1)
+    d1 = time.perf_counter() - t0
+    t0 = time.perf_counter()
+    P.run(0, n, X.SEED_L, cores)
+    dn = time.perf_counter() - t0
+    for name, c in (("spmd", G.cfg(G.SPMD, G.PL_STACK, 1, 256)), ("native_plain", G.cfg(G.NATIVE, G.PL_STACK, 1, 256)),
+                    ("csm", G.cfg(G.CSM, G.PL_STACK, 1, 256)), ("generic", G.cfg(G.GENERIC, G.PL_STACK, 1, 256))):
+        def f():
+            out.zero_()
+            G.gtr_xs_lookup(ctx, c, xs.tables, 0, n, X.SEED_L, out, None, stream)
+        ms = _time(torch, stream, f, 5)
+        res[name] = {"lookups_per_s": n / (ms * 1e-3), "ms": ms,
+                     "same_result_as_oracle": bool(np.array_equal(out.cpu().numpy(), o1))}
+    res["cpu_oracle_1core"] = {"lookups_per_s": n / d1, "cores": 1, "kind": "oracle", "sample": "full run"}
+    res["cpu_oracle_nproc"] = {"lookups_per_s": n / dn, "cores": cores, "kind": "oracle", "sample": "full run"}
+    del xs
+    torch.cuda.empty_cache()
+    return res
+
+
 # ---------------------------------------------------------------- reference arm
 def run_reference(a):
     ws = int(os.environ.get("WORLD_SIZE", "1"))
@@ -188,17 +290,19 @@ def run_gtr(a):
 
     # N > 1: the 18-u64 combine is fused into the lookup kernel's epilogue
     # (teams add into every rank's buffer over NVLink peer memory, then one
-    # device barrier; dist.PeerCombine); NCCL all_reduce only if the
-    # symmetric-memory rendezvous is unavailable on the box
-    pc, combine = None, None
+    # device barrier with a timeout; dist.PeerCombine) when every rank could
+    # set it up and its first result equals an NCCL all_reduce; otherwise --
+    # or with --combine nccl -- NCCL all_reduce.  All ranks decide together.
+    pc, combine, combine_check, nranks = None, "none (1 GPU)", None, ws
     if dist is not None:
         from paper_conf_cgo_hubercgtddcd22_b200.dist import PeerCombine
-        try:
-            pc = PeerCombine(dev)
+        pc, why = PeerCombine.create_all_or_none(dev, want=a.combine in ("auto", "fused"))
+        if pc is not None:
+            nranks = pc.nranks
             combine = "fused: team epilogue adds into every rank's buffer over NVLink peer memory + device barrier"
-        except Exception as e:  # noqa: BLE001 -- collective implementation choice, reported in the line
-            pc = None
-            combine = f"NCCL all_reduce (peer-memory rendezvous unavailable: {type(e).__name__})"
+        else:
+            combine = f"nccl: all_reduce(SUM) of 18 u64 ({why})" if a.combine != "nccl" else \
+                "nccl: all_reduce(SUM) of 18 u64 (--combine nccl)"
 
     def step():
         nonlocal out
@@ -214,19 +318,24 @@ def run_gtr(a):
     for _ in range(a.warmup):
         step()
     G.gtr_ctx_check(ctx, stream)
-    if pc is not None:
-        # one-time check of the fused combine against the NCCL all-reduce of
-        # this rank's own result (every box gpurun offers has one GPU, so the
-        # peer path is first exercised here); all ranks switch together
-        fused = out.clone()
+    if dist is not None:
+        # both combines on the same step, compared (also at N = 1 with
+        # GTR_BENCH_DIST=1): the fused result against the NCCL all-reduce of
+        # this rank's own lookups; all ranks switch to NCCL together if any differs
         loc = torch.zeros(18, dtype=torch.uint64, device=dev)
         G.gtr_xs_lookup(ctx, head, xs.tables, first, n, seed, loc, None, stream)
         combine_results(loc)
-        ok = torch.tensor([1 if torch.equal(fused.view(torch.int64), loc.view(torch.int64)) else 0], dtype=torch.int64, device=dev)
+        nccl_res = loc.cpu().numpy()
+        fused_res = out.cpu().numpy() if pc is not None else None
+        same = fused_res is None or bool(np.array_equal(fused_res, nccl_res))
+        ok = torch.tensor([1 if same else 0], dtype=torch.int64, device=dev)
         dist.all_reduce(ok, op=dist.ReduceOp.MIN)
-        if int(ok[0]) != 1:
+        combine_check = {"nccl_hash": int(nccl_res[0]),
+                         "fused_hash": int(fused_res[0]) if fused_res is not None else None,
+                         "identical_all_ranks": bool(int(ok[0]) == 1) if fused_res is not None else None}
+        if pc is not None and int(ok[0]) != 1:
             pc = None
-            combine = "NCCL all_reduce (fused peer-memory combine failed its check against NCCL)"
+            combine = "nccl: all_reduce(SUM) of 18 u64 (the fused peer-memory combine differed from NCCL)"
             step()
 
     # timed region: K steps, barrier + sync on both sides, CUDA events on the
@@ -285,7 +394,7 @@ def run_gtr(a):
     if not a.no_sweep:      # 180 GB HBM: the XS tables stay resident
         extra["sharded"] = sharded_apps(G, torch, ctx, rank, ws, dist, stream, dev)
     if rank == 0 and not a.no_sweep:
-        extra.update(sweeps(G, torch, ctx, xs, first, seed, stream))
+        extra.update(sweeps(G, torch, ctx, xs, first, seed, stream, cpu=(ws == 1 and not a.no_cpu_baseline)))
 
     # e2e through the public host-buffer entry point (H2D request, D2H results)
     h_out = torch.zeros(18, dtype=torch.uint64).pin_memory()
@@ -318,8 +427,8 @@ def run_gtr(a):
             "warmup": a.warmup, "ms_per_step": ms, "higher_is_better": True, "scaling": "weak",
             "vs_baseline": None, "dtype": "f64", "data": "synthetic",
             "config": {"workload": WORKLOAD, "variant": "SPMD + heap-to-stack + folding, thread_limit 256",
-                       "lookups_per_gpu": n, "parallelism": f"lookups sharded over {ws} GPU(s); combine of "
-                                                             f"hash+tallies: {combine}" if dist is not None else "1 GPU",
+                       "lookups_per_gpu": n, "parallelism": f"dp{ws}: lookups sharded over {ws} GPU(s)",
+                       "combine": combine, "nranks": nranks, "combine_check": combine_check,
                        "l2": "no flush: inputs 5.9 GB per GPU >> 126 MB L2 (index grid 5.7 GB)",
                        "table_setup_s": round(t_setup, 2)},
             "hash": int(res[0]), "hash_mod_999983": int(res[0] % 999983),
@@ -335,6 +444,7 @@ def run_gtr(a):
                             "stream sync; tables resident (uploaded once, table_setup_s)"},
             "gpu_launches": a.steps,
             "clocks": clk.summary(),
+            "host": host_info(),
         }
         line.update(extra)
         print(json.dumps(line), flush=True)
@@ -355,9 +465,11 @@ def _time(torch, stream, fn, reps):
     return a.elapsed_time(b) / reps
 
 
-def sweeps(G, torch, ctx, xs, first, seed, stream):
+def sweeps(G, torch, ctx, xs, first, seed, stream, cpu=True):
     """Per-mode lookups/s (same 17M lookups), the paper's variant ladder, and
-    fork/join ns per mode -- each checked for identical results."""
+    fork/join ns per mode -- each checked for identical results.  With `cpu`,
+    the oracle timed on the host cores beside every config (BASELINE.md
+    CPU-baseline plan)."""
     n = LOOKUPS_PER_GPU
     out = torch.zeros(18, dtype=torch.uint64, device="cuda")
     modes = {}
@@ -471,10 +583,16 @@ def sweeps(G, torch, ctx, xs, first, seed, stream):
         c = G.cfg(G.GENERIC, G.PL_STACK, 1, nt, num_teams=teams)
         row["generic_bcast_ns"] = _time(torch, stream, lambda: G.gtr_forkjoin(ctx, c, R, 2, 1, fo, stream), 2) \
             * 1e6 / R
+        if cpu:
+            row["cpu_oracle_host_team"] = oracle_fj(nt)
         fj[f"thread_limit_{nt}"] = row
     G.gtr_ctx_check(ctx, stream)
-    return {"modes": modes, "grid_types": grids, "history_and_sorted": f2, "ladder_spmd": ladder, "forkjoin": fj,
-            "su3": su3_sweep(G, torch, ctx, stream), "rsbench": rs_sweep(G, torch, ctx, stream)}
+    res = {"modes": modes, "grid_types": grids, "history_and_sorted": f2, "ladder_spmd": ladder, "forkjoin": fj,
+           "su3": su3_sweep(G, torch, ctx, stream), "rsbench": rs_sweep(G, torch, ctx, stream, cpu=cpu)}
+    if cpu:
+        res["su3"]["cpu_oracle"] = oracle_su3()
+        res["xs_small"] = xs_small_config(G, torch, ctx, stream)
+    return res
 
 
 def su3_sweep(G, torch, ctx, stream):
@@ -604,9 +722,9 @@ def sharded_apps(G, torch, ctx, rank, ws, dist, stream, dev):
     return res
 
 
-def rs_sweep(G, torch, ctx, stream, n=10_000_000):
+def rs_sweep(G, torch, ctx, stream, n=10_000_000, cpu=True):
     """Config 4: RSBench multipole lookups (355 nuclides, 10M lookups),
-    lookups/s per mode."""
+    lookups/s per mode (+ the oracle on the host cores, bounded sample)."""
     import gtr_inputs.rs as RS
     import gtr_inputs.xs as X
     from paper_conf_cgo_hubercgtddcd22_b200.problems import RsDevice
@@ -634,6 +752,13 @@ def rs_sweep(G, torch, ctx, stream, n=10_000_000):
                      "fallback_bytes_per_thread": G.gtr_ctx_fallback_high_water(ctx, reset=True, stream=stream)}
     G.gtr_ctx_check(ctx, stream)
     res["roofline_spmd"] = rs_roofline(G, torch, ctx, stream, 0, n, res["spmd"]["ms"])
+    if cpu:
+        orc, o_out = oracle_rs()
+        m = 100_000
+        out.zero_()
+        G.gtr_rs_lookup(ctx, G.cfg(G.SPMD, G.PL_STACK, 1, 128), dev.tables, 0, m, X.SEED_L, out, None, stream)
+        orc["same_result_as_gpu"] = bool(np.array_equal(out.cpu().numpy(), o_out))
+        res["cpu_oracle"] = orc
     return res
 
 

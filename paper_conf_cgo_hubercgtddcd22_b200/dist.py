@@ -75,15 +75,40 @@ class PeerCombine:
     (zero the other local slot, barrier on the current stream) -> the local
     slot holds the combined result."""
 
-    def __init__(self, device, group=None):
+    # a device barrier that waits longer than this traps (the process fails
+    # loudly) instead of hanging the job; one step takes ~17 ms
+    BARRIER_TIMEOUT_MS = 60_000
+
+    def __init__(self, device, group=None, timeout_ms=None):
         import torch.distributed as dist
         import torch.distributed._symmetric_memory as symm_mem
         g = group or dist.group.WORLD
+        self.timeout_ms = self.BARRIER_TIMEOUT_MS if timeout_ms is None else int(timeout_ms)
         self.buf = symm_mem.empty(36, dtype=torch.int64, device=device).view(2, 18)
         self.handle = symm_mem.rendezvous(self.buf, g.group_name)
+        self.nranks = int(self.handle.world_size)
         self.buf.zero_()
-        self.handle.barrier()
+        self.handle.barrier(0, self.timeout_ms)
         self.step = 0
+
+    @classmethod
+    def create_all_or_none(cls, device, group=None, want=True):
+        """Every rank tries to set the fused combine up; it is used only if it
+        succeeded on ALL ranks (a MIN all-reduce of the success flags), so the
+        ranks can never pick different combine paths.  Returns (PeerCombine or
+        None, reason)."""
+        import torch.distributed as dist
+        pc, why = None, None
+        if want:
+            try:
+                pc = cls(device, group)
+            except Exception as e:  # noqa: BLE001 -- any setup failure selects the NCCL path on every rank
+                why = f"{type(e).__name__}: {e}"[:160]
+        flag = torch.tensor([1 if pc is not None else 0], dtype=torch.int64, device=device)
+        dist.all_reduce(flag, op=dist.ReduceOp.MIN, group=group)
+        if int(flag[0]) != 1:
+            return None, why or ("not requested" if not want else "peer-memory setup failed on another rank")
+        return pc, None
 
     def ptrs(self):
         off = (self.step % 2) * 18 * 8
@@ -92,6 +117,6 @@ class PeerCombine:
     def finish(self):
         b = self.step % 2
         self.buf[1 - b].zero_()
-        self.handle.barrier()
+        self.handle.barrier(0, self.timeout_ms)
         self.step += 1
         return self.buf[b].view(torch.uint64)

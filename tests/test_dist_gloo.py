@@ -119,3 +119,35 @@ def test_sharded_rs_and_su3_equal_global(orc, ws):
     assert np.array_equal(rs, want)
     A, B = S.make_lattice(7 * ws, "random")                 # the global lattice
     assert np.array_equal(Cg, orc.su3_mat_nn(A, B).view(np.float64))
+
+
+def _worker_pc(rank, ws, port, want, q):
+    import torch.distributed as dist
+    from paper_conf_cgo_hubercgtddcd22_b200.dist import PeerCombine
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=ws)
+    pc, why = PeerCombine.create_all_or_none(torch.device("cpu"), want=want[rank])
+    q.put((rank, pc is None, why))
+    dist.destroy_process_group()
+
+
+@pytest.mark.parametrize("want", [(True, True), (True, False), (False, False)])
+def test_peer_combine_all_or_none(want):
+    """The fused combine is chosen by all ranks or by none (a MIN all-reduce of
+    the per-rank setup results): here peer-memory setup fails (CPU tensors) or
+    is not requested on some rank, and every rank must fall back to NCCL
+    together, with a reason, instead of deadlocking on mismatched paths."""
+    ws = len(want)
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_worker_pc, args=(r, ws, port, want, q)) for r in range(ws)]
+    for p in procs:
+        p.start()
+    res = sorted(q.get(timeout=120) for _ in range(ws))
+    for p in procs:
+        p.join(timeout=120)
+        assert p.exitcode == 0
+    assert all(none for _, none, _ in res)
+    assert all(why for _, _, why in res)
