@@ -77,6 +77,17 @@ int resolve(gtr_ctx *ctx, const gtr_launch_cfg *cfg, const void *fn, uint32_t de
     return GTR_OK;
 }
 
+// `teams distribute` chunk for n iterations: the kernel's chunk, or -- when
+// that leaves teams idle (n < chunk * teams) -- ceil(n / teams) rounded up to
+// a warp multiple, so the league is busy (results do not depend on it).
+inline uint32_t fit_chunk(uint64_t n, uint32_t chunk, int teams) {
+    if (teams < 1 || n >= (uint64_t)chunk * (uint64_t)teams) return chunk;
+    uint64_t c = (n + (uint64_t)teams - 1) / (uint64_t)teams;
+    c = (c + 31u) & ~(uint64_t)31u;
+    if (c < 32u) c = 32u;
+    return c < chunk ? (uint32_t)c : chunk;
+}
+
 template <class K> int fill_info(const void *fn, const Launch &L, int per_sm, gtr_variant_info *out) {
     cudaFuncAttributes a;
     GTR_CUDA_TRY(cudaFuncGetAttributes(&a, fn));

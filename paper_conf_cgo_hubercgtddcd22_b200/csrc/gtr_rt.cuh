@@ -38,6 +38,7 @@
 // without it they read the team/thread state in shared memory.
 #pragma once
 #include <cstdint>
+#include <cstring>
 #include <cuda_runtime.h>
 
 namespace gtr {
@@ -62,6 +63,18 @@ struct Cfg {
     static constexpr bool TSTATE = true;
     static_assert(NT_ % 32 == 0 && NT_ >= 32 && NT_ <= 1024 - (GENERIC_LIKE ? 32 : 0), "bad NT");
 };
+
+// Team-wide synchronisation of SPMD-mode code.  A team of one warp
+// (thread_limit 32: BLOCK == 32) is synchronised by __syncwarp -- the warp's
+// lanes are the whole team, and bar.warp.sync orders their shared-memory
+// accesses ("Team = warp" guards) -- instead of a CTA barrier.
+#ifndef GTR_WARP_TEAM
+#define GTR_WARP_TEAM 1   // 0: one-warp teams use CTA barriers and the shared broadcast slot (A/B)
+#endif
+template <class K> __device__ __forceinline__ void cta_sync() {
+    if constexpr (K::BLOCK == 32 && GTR_WARP_TEAM) __syncwarp();
+    else __syncthreads();
+}
 
 // Launch-time runtime parameters (host-filled, by value).
 struct RtParams {
@@ -135,7 +148,7 @@ template <class K> __device__ __forceinline__ void team_barrier() {
     if constexpr (K::GENERIC_LIKE)
         asm volatile("barrier.sync 1, %0;" ::"n"(K::BLOCK) : "memory");
     else
-        __syncthreads();
+        cta_sync<K>();
 }
 
 // `#pragma omp barrier` inside a parallel region: the region's threads only
@@ -160,7 +173,7 @@ template <class K> __device__ __forceinline__ void omp_barrier_full() {
     if constexpr (K::GENERIC_LIKE)
         asm volatile("barrier.sync 2, %0;" ::"n"(K::NT) : "memory");
     else
-        __syncthreads();
+        cta_sync<K>();
 }
 template <class K> __device__ __forceinline__ void omp_barrier() {
     if constexpr (K::FOLD) {
@@ -178,7 +191,7 @@ template <class K> __device__ __forceinline__ void omp_barrier() {
 // variable read by all threads is overwritten); generic: no-op (only the main
 // thread runs sequential code).
 template <class K> __device__ __forceinline__ void spmd_sync() {
-    if constexpr (K::MODE == SPMD) __syncthreads();
+    if constexpr (K::MODE == SPMD) cta_sync<K>();
 }
 
 // ---------------------------------------------------------------- queries
@@ -296,7 +309,7 @@ template <class K> __device__ __forceinline__ Role team_init(const RtParams &rp)
             g_ts.hwm_seen = 0;
             g_ts.rp = rp;
         }
-        __syncthreads();
+        cta_sync<K>();
         return Role::Main;
     }
 }
@@ -320,9 +333,9 @@ template <class K, class R> __device__ __forceinline__ void parallel(void *args,
             // one is a guarded side effect (its barriers only when it changes)
             const int n = region_threads<K>(num_threads_clause);
             if (n != g_ts.nthreads) {
-                __syncthreads();
+                cta_sync<K>();
                 if (threadIdx.x == 0) g_ts.nthreads = n;
-                __syncthreads();
+                cta_sync<K>();
             }
             tstate<K>().level = 1;
             if ((int)threadIdx.x < n) R::run(args);   // in place
@@ -330,7 +343,7 @@ template <class K, class R> __device__ __forceinline__ void parallel(void *args,
         } else {
             R::run(args);                        // in place, all threads
         }
-        __syncthreads();                         // join
+        cta_sync<K>();                           // join
     } else {
         static_assert(K::GENERIC_LIKE, "parallel() needs a runtime mode");
         if constexpr (K::MODE == CSM)
@@ -406,7 +419,7 @@ template <class K> __device__ __forceinline__ void team_deinit() {
 template <class K, class F> __device__ __forceinline__ void guarded(F &&f) {
     if constexpr (K::MODE == SPMD) {
         if (threadIdx.x == 0) f();
-        __syncthreads();
+        cta_sync<K>();
     } else {
         f();
     }
@@ -414,15 +427,27 @@ template <class K, class F> __device__ __forceinline__ void guarded(F &&f) {
 // A value produced in a guarded region, broadcast to all threads.  Default:
 // slot write -> barrier -> read -> barrier (the paper's 2 barriers,
 // P:687-688).  F_BCAST_1BAR: double-buffered slot, one barrier (`phase`
-// must alternate between consecutive calls).
+// must alternate between consecutive calls).  A one-warp team (thread_limit
+// 32): lane 0 computes, __shfl_sync broadcasts from its registers -- no
+// shared slot, no barrier.
 template <class K, class T, class F> __device__ __forceinline__ T guarded_bcast(F &&f, int phase = 0) {
     static_assert(sizeof(T) <= 8, "broadcast slot is 8 bytes");
-    if constexpr (K::MODE == SPMD) {
+    if constexpr (K::MODE == SPMD && K::BLOCK == 32 && GTR_WARP_TEAM) {
+        uint64_t w = 0;
+        if (threadIdx.x == 0) {
+            const T v = f();
+            memcpy(&w, &v, sizeof(T));
+        }
+        w = __shfl_sync(0xffffffffu, w, 0);
+        T v;
+        memcpy(&v, &w, sizeof(T));
+        return v;
+    } else if constexpr (K::MODE == SPMD) {
         int b = (K::FLAGS & F_BCAST_1BAR) ? (phase & 1) : 0;
         if (threadIdx.x == 0) *reinterpret_cast<T *>(&g_ts.bcast[b]) = f();
-        __syncthreads();
+        cta_sync<K>();
         T v = *reinterpret_cast<volatile T *>(&g_ts.bcast[b]);
-        if constexpr (!(K::FLAGS & F_BCAST_1BAR)) __syncthreads();
+        if constexpr (!(K::FLAGS & F_BCAST_1BAR)) cta_sync<K>();
         return v;
     } else {
         return f();
@@ -666,6 +691,12 @@ template <class K, class T, class Tag, bool RO = true> struct TeamLocal {
         else
             free_shared<K>(q, sizeof(T));
     }
+    // PRIVATE: the copy itself, never a stored pointer to it -- a member
+    // pointing into its own object keeps the whole object in local memory
+    // (SROA cannot split it), and every store to that stack slot then has to
+    // complete before the region's join barrier (measured: the SPMD
+    // heap-to-stack fork/join loop ran 151 ns per empty region at
+    // thread_limit 256, 3.5x the shared-memory form, all of it STL + BAR).
     T priv;
     T *p;
     __device__ __forceinline__ static T *static_slot() {
@@ -674,7 +705,6 @@ template <class K, class T, class Tag, bool RO = true> struct TeamLocal {
     }
     __device__ __forceinline__ TeamLocal() {
         if constexpr (PRIVATE) {
-            p = &priv;
         } else if constexpr (RUNTIME_ALLOC) {
             if constexpr (K::MODE == SPMD)
                 p = guarded_bcast<K, T *>([] { return alloc_one(); });
@@ -687,7 +717,7 @@ template <class K, class T, class Tag, bool RO = true> struct TeamLocal {
     __device__ __forceinline__ ~TeamLocal() {
         if constexpr (RUNTIME_ALLOC) {
             if constexpr (K::MODE == SPMD) {
-                __syncthreads();
+                cta_sync<K>();
                 if (threadIdx.x == 0) free_one(p);
             } else {
                 free_one(p);
@@ -696,10 +726,14 @@ template <class K, class T, class Tag, bool RO = true> struct TeamLocal {
     }
     // write by "the main thread": guarded in SPMD unless private
     template <class F> __device__ __forceinline__ void set(F &&f) {
-        if constexpr (PRIVATE || K::MODE != SPMD) f(*p);
+        if constexpr (PRIVATE) f(priv);
+        else if constexpr (K::MODE != SPMD) f(*p);
         else guarded<K>([&] { f(*p); });
     }
-    __device__ __forceinline__ T *get() { return p; }
+    __device__ __forceinline__ T *get() {
+        if constexpr (PRIVATE) return &priv;
+        else return p;
+    }
 };
 
 // ---------------------------------------------------------------- worksharing

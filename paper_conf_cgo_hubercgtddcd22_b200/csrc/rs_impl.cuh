@@ -501,7 +501,8 @@ template <class K> struct OpRt {
             GTR_CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, fn, K::BLOCK, L.dyn_smem));
             return fill_info<K>(fn, L, per_sm, a.info);
         }
-        a.P.chunk = (a.P.plain ? kLookupsPerThreadPerChunk : kBucketLookupsPerThread) * K::NT;
+        a.P.chunk = fit_chunk(a.P.n, (a.P.plain ? kLookupsPerThreadPerChunk : kBucketLookupsPerThread) * K::NT,
+                              L.teams);
         kernel_rt<K><<<L.teams, L.block, L.dyn_smem, a.stream>>>(a.P, L.rp);
         GTR_CUDA_TRY(cudaGetLastError());
         return GTR_OK;
