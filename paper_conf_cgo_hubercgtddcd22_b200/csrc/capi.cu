@@ -3,6 +3,7 @@
 #include <cstdlib>
 
 #include "gtr_internal.h"
+#include "tma.cuh"
 
 using namespace gtr;
 
@@ -41,6 +42,7 @@ extern "C" int gtr_ctx_create(int device, void *fallback_pool, uint64_t fallback
     }
     c->pool = static_cast<uint64_t *>(fallback_pool);
     c->pool_bytes = fallback_pool ? fallback_pool_bytes : 0;
+    c->spin_limit = GTR_DEFAULT_SPIN_LIMIT;
     *out = c;
     return GTR_OK;
 }
@@ -64,7 +66,44 @@ extern "C" int gtr_ctx_check(gtr_ctx *c, void *stream) {
     GTR_CUDA_TRY(cudaMemsetAsync(c->d_err, 0, sizeof(err), s));
     GTR_CUDA_TRY(cudaStreamSynchronize(s));
     if (err & ERR_HEAP) return GTR_EHEAP;
-    return GTR_EDEVICE;
+    return GTR_EDEVICE;     // ERR_HANG (watchdog), ERR_LIFO, ERR_DUP_ENERGY, ERR_BUILD
+}
+
+extern "C" int gtr_ctx_set_spin_limit(gtr_ctx *c, uint64_t polls) {
+    if (!c) return GTR_EINVAL;
+    c->spin_limit = polls ? polls : GTR_DEFAULT_SPIN_LIMIT;
+    return GTR_OK;
+}
+
+// Watchdog self-test: a kernel whose waits never complete (kind 0: a team's
+// software barrier expecting one more arrival than the team has; kind 1: an
+// mbarrier phase no one completes).  With the watchdog each wait gives up
+// after the context's spin limit, sets ERR_HANG and the kernel exits.
+namespace gtr {
+__global__ void k_watchdog_selftest(int32_t kind, RtParams rp) {
+    using K = Cfg<SPMD, PL_STACK, false, 64>;
+    team_init<K>(rp);
+    if (kind == 0) {
+        soft_barrier(K::NT + 1);                  // one arrival short: never completes
+    } else {
+        __shared__ uint64_t bar;
+        if (threadIdx.x == 0) tma::mbar_init(&bar);
+        __syncthreads();
+        tma::mbar_wait(&bar, 0, rp.spin_limit, rp.err, ERR_HANG);   // phase 0 never completes
+    }
+}
+}  // namespace gtr
+
+extern "C" int gtr_watchdog_selftest(gtr_ctx *c, int32_t kind, void *stream) {
+    if (!c || kind < 0 || kind > 1) return GTR_EINVAL;
+    using K = gtr::Cfg<gtr::SPMD, gtr::PL_STACK, false, 64>;
+    gtr::Launch L;
+    gtr_launch_cfg cfg = {2, 64, gtr::SPMD, gtr::PL_STACK, 0, 0, 0};
+    int st = gtr::resolve<K>(c, &cfg, reinterpret_cast<const void *>(&gtr::k_watchdog_selftest), 0, &L);
+    if (st) return st;
+    gtr::k_watchdog_selftest<<<L.teams, L.block, L.dyn_smem, static_cast<cudaStream_t>(stream)>>>(kind, L.rp);
+    GTR_CUDA_TRY(cudaGetLastError());
+    return GTR_OK;
 }
 
 extern "C" int gtr_ctx_fallback_high_water(gtr_ctx *c, uint64_t *bytes_out, int32_t reset, void *stream) {

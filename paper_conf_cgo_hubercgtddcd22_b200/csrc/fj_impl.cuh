@@ -104,8 +104,7 @@ template <class K, int BODY, int KMAX> __device__ __forceinline__ uint64_t team_
                     uint64_t x = g * (uint64_t)R + *ctr;
                     *ctr += 1;
                     return x;
-                },
-                (int)(r & 1));
+                });
         TeamLocal<K, Args, TagArgs> args;
         args.set([&](Args &x) {
             x.r = r;

@@ -15,7 +15,9 @@ struct gtr_ctx {
     uint64_t pool_bytes;
     uint32_t *d_err;       // device error word (+8: fallback high-water mark, u64)
     void *d_stage;         // 256 B staging buffer (e2e request / results)
+    uint64_t spin_limit;   // watchdog polls per spin-wait (gtr_ctx_set_spin_limit)
 };
+#define GTR_DEFAULT_SPIN_LIMIT (1ull << 26)
 
 namespace gtr {
 
@@ -74,6 +76,7 @@ int resolve(gtr_ctx *ctx, const gtr_launch_cfg *cfg, const void *fn, uint32_t de
     L->rp.pool_wpt = ctx->pool ? (ctx->pool_bytes / 8u) / hw : 0;
     L->rp.sm_stack_words = stack_words;
     L->rp.sm_stride_words = stride;
+    L->rp.spin_limit = ctx->spin_limit ? ctx->spin_limit : GTR_DEFAULT_SPIN_LIMIT;
     return GTR_OK;
 }
 

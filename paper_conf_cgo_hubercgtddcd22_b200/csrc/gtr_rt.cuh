@@ -45,7 +45,7 @@ namespace gtr {
 
 enum : int { GENERIC = 0, GENERIC_CASCADE = 1, CSM = 2, SPMD = 3, NATIVE = 4 };
 enum : int { PL_RUNTIME = 0, PL_GLOBAL = 1, PL_SHARED_STATIC = 2, PL_STACK = 3, PL_COALESCED = 4 };
-enum : uint32_t { ERR_HEAP = 1u, ERR_LIFO = 2u, ERR_DUP_ENERGY = 4u, ERR_BUILD = 8u };
+enum : uint32_t { ERR_HEAP = 1u, ERR_LIFO = 2u, ERR_DUP_ENERGY = 4u, ERR_BUILD = 8u, ERR_HANG = 16u };
 enum : int { F_BCAST_1BAR = 1, F_SEPARATE_GUARDS = 2 };
 
 // Compile-time kernel configuration.
@@ -84,7 +84,18 @@ struct RtParams {
     uint64_t pool_wpt;          // fallback capacity per hardware thread, 8-byte words
     uint32_t sm_stack_words;    // shared-memory stack capacity per thread (words)
     uint32_t sm_stride_words;   // per-thread stride of the stack (odd => no bank conflicts)
+    uint64_t spin_limit;        // watchdog: polls of a spin-wait before it gives up with ERR_HANG
 };
+
+// Watchdog of the runtime's spin-waits (software barrier, mbarrier waits,
+// the coalesced-free CAS loop): after `limit` polls the wait sets ERR_HANG in
+// the context's error word and returns -- the kernel finishes with results
+// declared invalid (gtr_ctx_check -> GTR_EDEVICE) instead of hanging the GPU.
+__device__ __forceinline__ bool spin_expired(uint64_t &polls, uint64_t limit, uint32_t *err) {
+    if (++polls < limit) return false;
+    atomicOr(err, (uint32_t)ERR_HANG);
+    return true;
+}
 
 typedef void (*RegionFn)(void *);
 
@@ -111,6 +122,8 @@ struct ThreadState {
     uint8_t nested;   // serialized nested parallel depth
     uint8_t level;    // SPMD: this thread's parallel level
     uint32_t gsp;     // global fallback stack top (words)
+    uint32_t bphase;  // F_BCAST_1BAR: broadcast slot of this thread's next guarded_bcast
+    uint32_t pad;
 };
 // PL_COALESCED only: per-lane + per-warp allocation state (after ThreadState)
 struct CoalState {
@@ -157,15 +170,22 @@ template <class K> __device__ __forceinline__ void team_barrier() {
 // A team smaller than NT (num_threads clause / ICV, non-folded variants):
 // named barrier 2 over its warps when it is whole warps, else a software
 // barrier in shared memory.  Serialized nested regions: a team of one.
+// Every access to the barrier's count and generation is atomic (the waiting
+// threads poll the generation the last arrival advances).
+__device__ __forceinline__ uint32_t atomic_load_shared(uint32_t *a) { return atomicOr(a, 0u); }
 static __device__ __noinline__ void soft_barrier(int n) {
     __threadfence_block();
-    const uint32_t gen = g_ts.sb_gen;
+    const uint32_t gen = atomic_load_shared(const_cast<uint32_t *>(&g_ts.sb_gen));
     if (atomicAdd(&g_ts.sb_count, 1u) == (uint32_t)n - 1u) {
-        g_ts.sb_count = 0;
+        atomicExch(&g_ts.sb_count, 0u);
         __threadfence_block();
-        g_ts.sb_gen = gen + 1u;
+        atomicAdd(const_cast<uint32_t *>(&g_ts.sb_gen), 1u);
     } else {
-        while (g_ts.sb_gen == gen) __nanosleep(32);
+        uint64_t polls = 0;
+        while (atomic_load_shared(const_cast<uint32_t *>(&g_ts.sb_gen)) == gen) {
+            if (spin_expired(polls, g_ts.rp.spin_limit, g_ts.rp.err)) break;
+            __nanosleep(32);
+        }
     }
     __threadfence_block();
 }
@@ -274,7 +294,7 @@ enum class Role { Main, Worker, Exit };
 // code, guarded).
 template <class K> __device__ __forceinline__ Role team_init(const RtParams &rp) {
     if constexpr (K::TSTATE) {
-        ThreadState z = {0, 0, 0, 0};
+        ThreadState z = {0, 0, 0, 0, 0, 0};
         tstate<K>() = z;
     }
     if constexpr (K::PL == 4 /*PL_COALESCED*/) {
@@ -426,11 +446,15 @@ template <class K, class F> __device__ __forceinline__ void guarded(F &&f) {
 }
 // A value produced in a guarded region, broadcast to all threads.  Default:
 // slot write -> barrier -> read -> barrier (the paper's 2 barriers,
-// P:687-688).  F_BCAST_1BAR: double-buffered slot, one barrier (`phase`
-// must alternate between consecutive calls).  A one-warp team (thread_limit
-// 32): lane 0 computes, __shfl_sync broadcasts from its registers -- no
-// shared slot, no barrier.
-template <class K, class T, class F> __device__ __forceinline__ T guarded_bcast(F &&f, int phase = 0) {
+// P:687-688).  F_BCAST_1BAR: double-buffered slot, one barrier -- every
+// call of the team alternates the slot (a per-thread phase; all threads make
+// the same calls), so thread 0's write of slot b in call k+2 follows call
+// k+1's barrier, which every reader of call k's slot b passed after reading
+// (a caller-chosen phase let the runtime's own broadcasts, e.g. a TeamLocal
+// pointer, reuse the slot a value was still being read from).  A one-warp
+// team (thread_limit 32): lane 0 computes, __shfl_sync broadcasts from its
+// registers -- no shared slot, no barrier.
+template <class K, class T, class F> __device__ __forceinline__ T guarded_bcast(F &&f) {
     static_assert(sizeof(T) <= 8, "broadcast slot is 8 bytes");
     if constexpr (K::MODE == SPMD && K::BLOCK == 32 && GTR_WARP_TEAM) {
         uint64_t w = 0;
@@ -443,7 +467,11 @@ template <class K, class T, class F> __device__ __forceinline__ T guarded_bcast(
         memcpy(&v, &w, sizeof(T));
         return v;
     } else if constexpr (K::MODE == SPMD) {
-        int b = (K::FLAGS & F_BCAST_1BAR) ? (phase & 1) : 0;
+        int b = 0;
+        if constexpr ((K::FLAGS & F_BCAST_1BAR) != 0) {
+            b = (int)(tstate<K>().bphase & 1u);
+            tstate<K>().bphase ^= 1u;
+        }
         if (threadIdx.x == 0) *reinterpret_cast<T *>(&g_ts.bcast[b]) = f();
         cta_sync<K>();
         T v = *reinterpret_cast<volatile T *>(&g_ts.bcast[b]);
@@ -466,13 +494,11 @@ template <class K> __device__ __forceinline__ void set_num_threads(int n) {
 // that is exhausted, ERR_HEAP and a per-CTA sink (results declared invalid).
 __device__ __align__(16) static uint64_t g_sink_dummy;
 // Fallback high-water mark: the global atomic only when this team has not
-// yet reported that many bytes (a racy but monotone filter: a few atomics
-// per team instead of one per allocation).
+// yet reported that many bytes (a per-team shared-memory atomicMax filters:
+// a few global atomics per team instead of one per allocation).
 __device__ __forceinline__ void note_fallback(const RtParams &rp, uint32_t bytes) {
-    if (bytes > g_ts.hwm_seen) {
-        g_ts.hwm_seen = bytes;
+    if (atomicMax(const_cast<uint32_t *>(&g_ts.hwm_seen), bytes) < bytes)   // shared atomic: the team's filter
         atomicMax(rp.hwm, (unsigned long long)bytes);
-    }
 }
 template <class K> __device__ __noinline__ void *alloc_shared(uint32_t bytes) {
     const uint32_t words = (bytes + 7u) >> 3;
@@ -538,21 +564,28 @@ template <class K> __device__ __noinline__ void *alloc_coalesced(uint32_t words,
     }
     uint64_t *p = nullptr;
     int k = -1;
+    // the converged warp meets here: each lane's accesses to frames it
+    // released earlier are ordered before the frame is handed out again
+    // (bar.warp.sync; the frame atomics alone do not order plain accesses)
+    __syncwarp();
     if ((threadIdx.x & 31u) == 0) {
         CoalState *W = warp_states<K>();
         const uint32_t cap = min(32u * rp.sm_stride_words, 32767u);
         const uint32_t wbase = threadIdx.x & ~31u;
-        k = (int)W[0].nframes;
+        // the warp stack is also popped by lanes releasing frames (possibly
+        // diverged, interleaved with this allocation): atomics throughout
+        k = (int)atomic_load_shared(&W[0].nframes);
         uint32_t glob = 0;
+        const uint32_t wtop = atomic_load_shared(&W[0].wtop), wgtop = atomic_load_shared(&W[0].wgtop);
         if (k >= 32 || words > 32767u) {
             k = -1;
-        } else if (W[0].wtop + words <= cap) {
-            p = sm_stack_base<K>() + (size_t)wbase * rp.sm_stride_words + W[0].wtop;
-            W[0].wtop += words;
-        } else if (rp.pool != nullptr && (uint64_t)W[0].wgtop + words <= 32u * half) {
-            p = rp.pool + ((uint64_t)blockIdx.x * K::BLOCK + wbase) * half + W[0].wgtop;
-            W[0].wgtop += words;
-            note_fallback(rp, W[0].wgtop * 8u / 32u);   // warp SoA: per lane
+        } else if (wtop + words <= cap) {
+            p = sm_stack_base<K>() + (size_t)wbase * rp.sm_stride_words + wtop;
+            atomicAdd(&W[0].wtop, words);
+        } else if (rp.pool != nullptr && (uint64_t)wgtop + words <= 32u * half) {
+            p = rp.pool + ((uint64_t)blockIdx.x * K::BLOCK + wbase) * half + wgtop;
+            atomicAdd(&W[0].wgtop, words);
+            note_fallback(rp, (wgtop + words) * 8u / 32u);   // warp SoA: per lane
             glob = 0x8000u;
         } else {
             k = -1;
@@ -561,9 +594,9 @@ template <class K> __device__ __noinline__ void *alloc_coalesced(uint32_t words,
             atomicOr(rp.err, (uint32_t)ERR_HEAP);
             p = &g_sink_dummy;
         } else {
-            W[k].frame = (32u << 16) | glob | words;
+            atomicExch(&W[k].frame, (32u << 16) | glob | words);
             __threadfence_block();
-            W[0].nframes = (uint32_t)k + 1u;
+            atomicExch(&W[0].nframes, (uint32_t)k + 1u);
         }
     }
     fk = __shfl_sync(0xffffffffu, k, 0);
@@ -579,10 +612,12 @@ template <class K> __device__ __noinline__ void free_coalesced(void *p, uint32_t
     __threadfence_block();                                // this lane's uses happen before release
     const uint32_t old = atomicSub(&W[fk].frame, 1u << 16);
     if ((old >> 16) != 1u) return;                        // other lanes still use frame fk
+    uint64_t polls = 0;
     for (;;) {                                            // pop fully released frames
-        const uint32_t n = *reinterpret_cast<volatile uint32_t *>(&W[0].nframes);
+        if (spin_expired(polls, g_ts.rp.spin_limit, g_ts.rp.err)) break;
+        const uint32_t n = atomic_load_shared(&W[0].nframes);
         if (n == 0) break;
-        const uint32_t f = *reinterpret_cast<volatile uint32_t *>(&W[n - 1].frame);
+        const uint32_t f = atomic_load_shared(&W[n - 1].frame);
         if ((f >> 16) != 0u) break;
         if (atomicCAS(&W[0].nframes, n, n - 1) != n) continue;
         if (f & 0x8000u) atomicSub(&W[0].wgtop, f & 0x7fffu);

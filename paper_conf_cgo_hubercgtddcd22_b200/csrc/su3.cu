@@ -35,7 +35,7 @@ template <int NT> __global__ void __launch_bounds__(NT) kernel_native(Params P) 
 // NATIVE, tile-streamed (GTR_F_TMA): persistent CTAs; thread 0 streams
 // 16-site A tiles into a double buffer with bulk asynchronous copies (TMA) and
 // C tiles back; the CTA computes each tile from shared memory.
-template <int NT> __global__ void __launch_bounds__(NT) kernel_native_tma(Params P) {
+template <int NT> __global__ void __launch_bounds__(NT) kernel_native_tma(Params P, uint32_t *err, uint64_t spin_limit) {
     extern __shared__ __align__(128) uint8_t dyn[];
     TileBuf &tb = *reinterpret_cast<TileBuf *>(dyn);
     const int64_t ntiles = (P.sites + kTileSites - 1) / kTileSites;
@@ -61,7 +61,7 @@ template <int NT> __global__ void __launch_bounds__(NT) kernel_native_tma(Params
             tma::store_wait_read();
         }
         __syncthreads();
-        tma::mbar_wait(&tb.bar[i & 1], (uint32_t)((i >> 1) & 1));
+        tma::mbar_wait(&tb.bar[i & 1], (uint32_t)((i >> 1) & 1), spin_limit, err, ERR_HANG);
         const double2 *At = tb.a[i & 1];
         const int total = (int)tile_sites(t) * 36;
         for (int q = threadIdx.x; q < total; q += NT) {
@@ -96,7 +96,8 @@ template <int NT> int run_native_tma(LaunchArgs &a) {
     L.dyn_smem = smem;
     L.teams = a.cfg->num_teams > 0 ? a.cfg->num_teams : per_sm * a.ctx->num_sms;
     if (a.info) return fill_info<Cfg<NATIVE, PL_STACK, true, NT>>(fn, L, per_sm, a.info);
-    for (int32_t it = 0; it < a.iters; it++) kernel_native_tma<NT><<<L.teams, NT, smem, a.stream>>>(a.P);
+    for (int32_t it = 0; it < a.iters; it++)
+        kernel_native_tma<NT><<<L.teams, NT, smem, a.stream>>>(a.P, a.ctx->d_err, a.ctx->spin_limit);
     GTR_CUDA_TRY(cudaGetLastError());
     return GTR_OK;
 }

@@ -100,7 +100,7 @@ template <class K> struct TileRegion {
     static __device__ void run(void *a) {
         const TileArgs *t = static_cast<const TileArgs *>(a);
         TileBuf &tb = tile_buf<K>();
-        tma::mbar_wait(&tb.bar[t->buf], t->parity);             // A tile landed
+        tma::mbar_wait(&tb.bar[t->buf], t->parity, g_ts.rp.spin_limit, g_ts.rp.err, ERR_HANG);   // A tile landed
         const double2 *At = tb.a[t->buf];
         for_static<K>(0, (int64_t)t->ns * 36, [&](int64_t q) {
             const int site = (int)(q / 36), e = (int)(q - site * 36);

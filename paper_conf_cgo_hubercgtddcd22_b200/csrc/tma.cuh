@@ -30,15 +30,29 @@ __device__ __forceinline__ void load_async(void *dst, const void *src, uint32_t 
                  "l"(src), "r"(bytes), "r"(smem_addr(bar))
                  : "memory");
 }
-// consumer: wait until the barrier completed the phase with parity `parity`
-__device__ __forceinline__ void mbar_wait(uint64_t *bar, uint32_t parity) {
+// consumer: wait until the barrier completed the phase with parity `parity`.
+// Watchdog: after `limit` unsuccessful try_waits (each suspends for a
+// hardware-chosen time) set `hang_bit` in *err and return -- the data is then
+// invalid and the host sees the error (gtr_ctx_check).
+__device__ __forceinline__ bool mbar_try_wait(uint64_t *bar, uint32_t parity) {
+    uint32_t ok;
     asm volatile(
-        "{\n\t.reg .pred p;\n"
-        "WAIT_%=:\n\t"
-        "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n\t"
-        "@!p bra WAIT_%=;\n}" ::"r"(smem_addr(bar)),
-        "r"(parity)
+        "{\n\t.reg .pred p;\n\t"
+        "mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n\t"
+        "selp.u32 %0, 1, 0, p;\n}"
+        : "=r"(ok)
+        : "r"(smem_addr(bar)), "r"(parity)
         : "memory");
+    return ok != 0;
+}
+__device__ __forceinline__ void mbar_wait(uint64_t *bar, uint32_t parity, uint64_t limit, uint32_t *err,
+                                          uint32_t hang_bit) {
+    for (uint64_t polls = 0; !mbar_try_wait(bar, parity);) {
+        if (++polls >= limit) {
+            atomicOr(err, hang_bit);
+            return;
+        }
+    }
 }
 // order this thread's generic-proxy shared-memory writes before later async-
 // proxy reads (a bulk store issued after a barrier)

@@ -92,6 +92,8 @@ _proto = {
     "gtr_ctx_destroy": (_i, [_vp]),
     "gtr_ctx_check": (_i, [_vp, _vp]),
     "gtr_ctx_fallback_high_water": (_i, [_vp, C.POINTER(C.c_uint64), C.c_int32, _vp]),
+    "gtr_ctx_set_spin_limit": (_i, [_vp, _u64]),
+    "gtr_watchdog_selftest": (_i, [_vp, C.c_int32, _vp]),
     "gtr_query_variant": (_i, [_i, _P(gtr_launch_cfg), _P(gtr_variant_info)]),
     "gtr_forkjoin": (_i, [_vp, _P(gtr_launch_cfg), _i64, C.c_int32, C.c_int32, _vp, _vp]),
     "gtr_barrier_floor": (_i, [_vp, _P(gtr_launch_cfg), _i64, _vp, _vp]),
@@ -178,6 +180,16 @@ def gtr_ctx_fallback_high_water(ctx, reset=False, stream=None):
     _check("gtr_ctx_fallback_high_water", _lib.gtr_ctx_fallback_high_water(ctx, C.byref(v), 1 if reset else 0,
                                                                             _stream(stream)))
     return int(v.value)
+
+
+def gtr_ctx_set_spin_limit(ctx, polls):
+    """Watchdog: polls of a runtime spin-wait before it sets the hang bit (0: default)."""
+    return _check("gtr_ctx_set_spin_limit", _lib.gtr_ctx_set_spin_limit(ctx, polls))
+
+
+def gtr_watchdog_selftest(ctx, kind, stream=None):
+    """Enqueue a kernel whose waits never complete (0: software barrier, 1: mbarrier)."""
+    return _check("gtr_watchdog_selftest", _lib.gtr_watchdog_selftest(ctx, kind, _stream(stream)))
 
 
 def gtr_query_variant(kernel, launch_cfg):

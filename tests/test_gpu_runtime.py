@@ -103,3 +103,23 @@ def test_fig7_separate_guards_same_result(G, ctx, orc, pl):
         G.gtr_semantics(ctx, G.cfg(G.SPMD, pl, 1, 64, num_teams=6, flags=flags), 4, out, out.numel())
         G.gtr_ctx_check(ctx)
         assert np.array_equal(out.cpu().numpy(), want)
+
+
+@pytest.mark.parametrize("kind", (0, 1), ids=("soft_barrier", "mbarrier"))
+def test_watchdog_trips(G, ctx, kind):
+    """A kernel whose wait can never complete (a software barrier one arrival
+    short; an mbarrier phase nobody completes) finishes once the watchdog's
+    spin limit is reached and reports the hang through the error word
+    (GTR_EDEVICE) instead of hanging the GPU; the context is usable after."""
+    G.gtr_ctx_set_spin_limit(ctx, 20000)
+    try:
+        G.gtr_watchdog_selftest(ctx, kind)
+        with pytest.raises(G.GtrError, match="device-side"):
+            G.gtr_ctx_check(ctx)
+    finally:
+        G.gtr_ctx_set_spin_limit(ctx, 0)
+    G.gtr_ctx_check(ctx)                         # cleared
+    out = torch.zeros(4, dtype=torch.uint64, device="cuda")
+    G.gtr_forkjoin(ctx, G.cfg(G.SPMD, G.PL_STACK, 1, 128, num_teams=4), 10, 0, 1, out)
+    G.gtr_ctx_check(ctx)
+    assert (out.cpu().numpy() == 10).all()
