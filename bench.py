@@ -482,6 +482,8 @@ def sweeps(G, torch, ctx, xs, first, seed, stream, cpu=True):
             if not tag:     # generic modes run thread_limit + 32 threads: 128 fits more teams/SM
                 variants.append((name + "_t128", G.cfg(m, G.PL_STACK, 1, 128, flags=sched)))
     variants.insert(0, ("native_plain", G.cfg(G.NATIVE, G.PL_STACK, 1, 256)))
+    # the CUDA watermark of the bucketed schedule (plain CUDA, no runtime)
+    variants.insert(1, ("native_bucketed", G.cfg(G.NATIVE, G.PL_STACK, 1, 256, flags=G.F_NATIVE_BUCKETED)))
     for name, c in variants:
         def f():
             out.zero_()
@@ -493,6 +495,14 @@ def sweeps(G, torch, ctx, xs, first, seed, stream, cpu=True):
         modes[name] = {"lookups_per_s": n / (ms * 1e-3), "ms": ms, "regs": info["regs"],
                        "static_smem": info["static_smem"], "dyn_smem": info["dyn_smem"],
                        "teams_per_sm": info["teams_per_sm"], "same_result": bool(np.array_equal(r, ref))}
+    # the paper's "OpenMP as a fraction of CUDA" (its V100: XS 71%,
+    # RS 98%): each runtime mode against the CUDA kernel of the same schedule
+    rate = {k: v["lookups_per_s"] for k, v in modes.items()}
+    modes["fraction_of_cuda"] = {
+        "bucketed_schedule": {m: rate[m] / rate["native_bucketed"] for m in ("spmd", "csm", "cascade", "generic")},
+        "paper_plain_schedule": {m: rate[m + "_plain"] / rate["native_plain"]
+                                 for m in ("spmd", "csm", "cascade", "generic")},
+        "paper_v100": {"xsbench_llvm_dev_vs_cuda": 0.71}}
     # XSBench's other acceleration structures, same lookups
     grids = {}
     import gtr_inputs.xs as X
@@ -733,6 +743,7 @@ def rs_sweep(G, torch, ctx, stream, n=10_000_000, cpu=True):
     res = {"workload": f"355 nuclides, ~1000 poles / 100 windows each, {n} lookups"}
     ref = None
     for name, c in [("native_plain", G.cfg(G.NATIVE, G.PL_STACK, 1, 128)),
+                    ("native_bucketed", G.cfg(G.NATIVE, G.PL_STACK, 1, 128, flags=G.F_NATIVE_BUCKETED)),
                     ("spmd", G.cfg(G.SPMD, G.PL_STACK, 1, 128)),
                     ("spmd_plain", G.cfg(G.SPMD, G.PL_STACK, 1, 128, flags=G.F_PLAIN)),
                     ("csm", G.cfg(G.CSM, G.PL_STACK, 1, 128)),
@@ -751,6 +762,11 @@ def rs_sweep(G, torch, ctx, stream, n=10_000_000, cpu=True):
                      "same_result": bool(np.array_equal(r, ref)),
                      "fallback_bytes_per_thread": G.gtr_ctx_fallback_high_water(ctx, reset=True, stream=stream)}
     G.gtr_ctx_check(ctx, stream)
+    rate = {k: v["lookups_per_s"] for k, v in res.items() if isinstance(v, dict)}
+    res["fraction_of_cuda"] = {
+        "bucketed_schedule": {m: rate[m] / rate["native_bucketed"] for m in ("spmd", "csm", "generic")},
+        "paper_plain_schedule": {m: rate[m + "_plain"] / rate["native_plain"] for m in ("spmd", "generic")},
+        "paper_v100": {"rsbench_llvm_dev_vs_cuda": 0.98}}
     res["roofline_spmd"] = rs_roofline(G, torch, ctx, stream, 0, n, res["spmd"]["ms"])
     if cpu:
         orc, o_out = oracle_rs()

@@ -36,10 +36,34 @@ template <int NT> int run_native(LaunchArgs &a) {
     return GTR_OK;
 }
 
+template <int NT> int run_native_bucketed(LaunchArgs &a) {
+    using KN = Cfg<NATIVE, PL_STACK, true, NT>;
+    const void *fn = reinterpret_cast<const void *>(&kernel_native_bucketed<KN>);
+    const uint32_t smem = (uint32_t)sizeof(ChunkBuf<KN>);
+    GTR_CUDA_TRY(cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+    int per_sm = 0;
+    GTR_CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, fn, NT, smem));
+    if (per_sm < 1) return GTR_EINVAL;
+    Launch L;
+    L.block = NT;
+    L.dyn_smem = smem;
+    L.teams = a.cfg->num_teams > 0 ? a.cfg->num_teams : per_sm * a.ctx->num_sms;
+    if (a.info) return fill_info<KN>(fn, L, per_sm, a.info);
+    a.P.chunk = fit_chunk(a.P.n, kBucketLookupsPerThread * NT, L.teams);
+    kernel_native_bucketed<KN><<<L.teams, NT, smem, a.stream>>>(a.P);
+    GTR_CUDA_TRY(cudaGetLastError());
+    return GTR_OK;
+}
+
 inline int launch(LaunchArgs &a) {
     const gtr_launch_cfg *c = a.cfg;
     if (!valid_cfg(c)) return GTR_EINVAL;
     a.P.plain = (c->flags & GTR_F_PLAIN) ? 1 : 0;
+    if (c->mode == NATIVE && (c->flags & GTR_F_NATIVE_BUCKETED)) {
+        if (a.P.plain) return GTR_EINVAL;
+        if (c->thread_limit == 128) return run_native_bucketed<128>(a);
+        return GTR_EUNSUPPORTED;
+    }
     if (c->mode == NATIVE) {
         if (c->thread_limit == 128) return run_native<128>(a);
         if (c->thread_limit == 256) return run_native<256>(a);

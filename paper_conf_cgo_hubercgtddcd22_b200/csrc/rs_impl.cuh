@@ -377,6 +377,7 @@ template <class K> struct ChunkBuf {
     unsigned int next;
 };
 template <class K> __device__ __forceinline__ ChunkBuf<K> &chunk_buf() {
+    if constexpr (K::MODE == NATIVE) return *reinterpret_cast<ChunkBuf<K> *>(g_dyn);   // no runtime state
     const uint32_t off = tstate_bytes<K>() + (uint32_t)K::BLOCK * g_ts.rp.sm_stride_words * 8u;
     return *reinterpret_cast<ChunkBuf<K> *>(g_dyn + ((off + 15u) & ~15u));
 }
@@ -476,6 +477,46 @@ template <class K> __global__ void __launch_bounds__(K::BLOCK, K::NT == 128 ? (K
     if constexpr (K::MODE == SPMD) flush(g_tally, g_p.out, threadIdx.x, K::NT);
     else flush(g_tally, g_p.out, 0, 1);
     team_deinit<K>();
+}
+
+// The CUDA watermark of the bucketed schedule (GTR_F_NATIVE_BUCKETED), as in
+// xs_impl.cuh: the team program as a plain CUDA kernel, no runtime.
+template <class K>
+__global__ void __launch_bounds__(K::NT, K::NT == 128 ? GTR_RS_MINB : 1) kernel_native_bucketed(Params P) {
+    static_assert(K::MODE == NATIVE, "plain CUDA");
+    if (threadIdx.x == 0) {
+        g_p = P;
+        for (int k = 0; k < 17; k++) g_tally[k] = 0;
+    }
+    __syncthreads();
+    const uint64_t n = g_p.n, ch = g_p.chunk;
+    const uint64_t nchunks = (n + ch - 1) / ch;
+    ChunkBuf<K> &b = chunk_buf<K>();
+    __shared__ Chunk chunk;
+    for (uint64_t c = blockIdx.x; c < nchunks; c += gridDim.x) {
+        if (threadIdx.x == 0) {
+            chunk.base = g_p.first + c * ch;
+            chunk.count = (c * ch + ch <= n) ? ch : n - c * ch;
+            for (int m = 0; m < 12; m++) b.cnt[m] = 0;
+            b.next = 0;
+        }
+        __syncthreads();
+        SampleRegion<K>::run(&chunk);
+        __syncthreads();
+        if (threadIdx.x == 0) {
+            uint32_t off = 0;
+            for (int m = 0; m < 12; m++) {
+                b.cur[m] = off;
+                off += b.cnt[m];
+            }
+        }
+        __syncthreads();
+        ScatterRegion<K>::run(&chunk);
+        __syncthreads();
+        BucketRegion<K>::run(&chunk);
+        __syncthreads();
+    }
+    flush(g_tally, g_p.out, threadIdx.x, K::NT);
 }
 
 struct LaunchArgs {

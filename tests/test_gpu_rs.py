@@ -165,7 +165,7 @@ def test_rs_full_size_bench_launch(G, ctx, orc):
 
 # ---------------------------------------------------------------- edge cases
 EDGE_CFGS = [(3, 3, 1, 128, 0), (3, 0, 0, 128, 0), (2, 3, 1, 128, 0), (0, 2, 0, 128, 0), (1, 4, 0, 128, 0),
-             (3, 3, 1, 128, 4), (4, 3, 1, 128, 0), (4, 3, 1, 256, 0)]
+             (3, 3, 1, 128, 4), (4, 3, 1, 128, 0), (4, 3, 1, 256, 0), (4, 3, 1, 128, 32)]
 
 
 def _edge_run(G, ctx, orc, t, first, n, seed, cfgs=EDGE_CFGS, wide=(True, False)):
@@ -283,3 +283,11 @@ def test_rs_energy_exactly_one(G, ctx, orc):
     assert E == 1.0
     t = RS.make_tables(avg_poles=100, avg_windows=10, seed=5)
     _edge_run(G, ctx, orc, t, 0, 64, seed)
+
+
+def test_rs_native_bucketed(G, ctx, dev, dev_narrow, rs):
+    """GTR_F_NATIVE_BUCKETED: the bucketed schedule as plain CUDA -- same
+    lookups (R-RS-tol), several chunks per team and the default league."""
+    for d in (dev, dev_narrow):
+        _check(G, ctx, d, rs, G.cfg(G.NATIVE, G.PL_STACK, 1, 128, flags=G.F_NATIVE_BUCKETED))
+        _check(G, ctx, d, rs, G.cfg(G.NATIVE, G.PL_STACK, 1, 128, num_teams=TEAMS_RS, flags=G.F_NATIVE_BUCKETED))

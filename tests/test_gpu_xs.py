@@ -438,3 +438,37 @@ def test_large_config_bench_launch(G, ctx, orc):
     o2, ov = P.run(first, m, X.SEED_L, 8, verify=True)
     out, v = _run(G, ctx, dev, G.cfg(G.SPMD, G.PL_STACK, 1, 256), first, m)
     _assert_same(out, v, o2, ov)
+
+
+# ---------------------------------------------------------------- CUDA watermark of the bucketed schedule
+@pytest.mark.parametrize("nt", (128, 256))
+def test_native_bucketed_bit_exact(G, ctx, dev_small, small, nt):
+    """GTR_F_NATIVE_BUCKETED: the bucketed/staged schedule as a plain CUDA
+    kernel (no runtime) -- bit-identical lookups, also over a few teams with
+    several chunks each and with ragged requests."""
+    t, P, o_out, o_v, n = small
+    c = G.cfg(G.NATIVE, G.PL_STACK, 1, nt, flags=G.F_NATIVE_BUCKETED)
+    _assert_same(*_run(G, ctx, dev_small, c, 0, n), o_out, o_v)
+    c2 = G.cfg(G.NATIVE, G.PL_STACK, 1, nt, num_teams=3, flags=G.F_NATIVE_BUCKETED)
+    _assert_same(*_run(G, ctx, dev_small, c2, 0, n), o_out, o_v)
+    for first, m in ((7, 1), (31337, 4097), (3, 12345)):
+        _assert_same(*_run(G, ctx, dev_small, c2, first, m), *P.run(first, m, X.SEED_L, 4, verify=True))
+
+
+def test_native_bucketed_sorted_and_grids(G, ctx, dev_small, dev_grid, small):
+    t, P, o_out, o_v, n = small
+    c = G.cfg(G.NATIVE, G.PL_STACK, 1, 256, flags=G.F_NATIVE_BUCKETED)
+    out, v = _run_sorted(G, ctx, dev_small, c, 0, n)
+    _assert_same(out, v, o_out, o_v)
+    gt, dev = dev_grid
+    out, v = _run(G, ctx, dev, c, 0, n)
+    assert np.array_equal(out, o_out)
+    assert np.array_equal(v["macro"].view(np.uint64), o_v["macro"].view(np.uint64))
+
+
+def test_native_bucketed_rejects_plain_and_history(G, ctx, dev_small):
+    out = torch.zeros(18, dtype=torch.uint64, device="cuda")
+    for fl in (G.F_PLAIN, G.F_HISTORY):
+        with pytest.raises(G.GtrError):
+            G.gtr_xs_lookup(ctx, G.cfg(G.NATIVE, G.PL_STACK, 1, 256, flags=G.F_NATIVE_BUCKETED | fl),
+                            dev_small.tables, 0, 1000, X.SEED_L, out)

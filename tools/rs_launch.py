@@ -18,6 +18,7 @@ from paper_conf_cgo_hubercgtddcd22_b200.problems import RsDevice  # noqa: E402
 
 VARIANTS = {
     "native": G.cfg(G.NATIVE, G.PL_STACK, 1, 128),
+    "native_bucketed": G.cfg(G.NATIVE, G.PL_STACK, 1, 128, flags=G.F_NATIVE_BUCKETED),
     "spmd": G.cfg(G.SPMD, G.PL_STACK, 1, 128),
     "spmd_plain": G.cfg(G.SPMD, G.PL_STACK, 1, 128, flags=G.F_PLAIN),
     "csm": G.cfg(G.CSM, G.PL_STACK, 1, 128),

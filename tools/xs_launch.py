@@ -17,6 +17,11 @@ from paper_conf_cgo_hubercgtddcd22_b200.problems import XsDevice  # noqa: E402
 
 VARIANTS = {
     "native": G.cfg(G.NATIVE, G.PL_STACK, 1, 256),
+    "native_bucketed": G.cfg(G.NATIVE, G.PL_STACK, 1, 256, flags=G.F_NATIVE_BUCKETED),
+    "native_2teams": G.cfg(G.NATIVE, G.PL_STACK, 1, 256, num_teams=296),   # the SPMD kernel's occupancy
+    "spmd_plain_t128": G.cfg(G.SPMD, G.PL_STACK, 1, 128, flags=G.F_PLAIN),
+    "native_t128": G.cfg(G.NATIVE, G.PL_STACK, 1, 128),
+    "csm_plain": G.cfg(G.CSM, G.PL_STACK, 1, 256, flags=G.F_PLAIN),
     "spmd": G.cfg(G.SPMD, G.PL_STACK, 1, 256),
     "spmd128": G.cfg(G.SPMD, G.PL_STACK, 1, 128),
     "spmd_shared": G.cfg(G.SPMD, G.PL_SHARED_STATIC, 1, 256),
