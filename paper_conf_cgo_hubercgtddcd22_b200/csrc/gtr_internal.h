@@ -91,6 +91,20 @@ inline uint32_t fit_chunk(uint64_t n, uint32_t chunk, int teams) {
     return c < chunk ? (uint32_t)c : chunk;
 }
 
+// Balanced `teams distribute` chunk: the fewest rounds the kernel's chunk
+// allows (ceil(n / (chunk * teams))), each as full as possible -- the last
+// round of equal chunks otherwise leaves most teams idle (10M RS lookups in
+// chunks of 4096 over 592 teams: 4.1 rounds run as 5).
+inline uint32_t balanced_chunk(uint64_t n, uint32_t chunk, int teams) {
+    if (teams < 1 || n == 0) return chunk;
+    const uint64_t per_round = (uint64_t)chunk * (uint64_t)teams;
+    const uint64_t rounds = (n + per_round - 1) / per_round;
+    uint64_t c = (n + rounds * (uint64_t)teams - 1) / (rounds * (uint64_t)teams);
+    c = (c + 31u) & ~(uint64_t)31u;
+    if (c < 32u) c = 32u;
+    return c < chunk ? (uint32_t)c : chunk;
+}
+
 template <class K> int fill_info(const void *fn, const Launch &L, int per_sm, gtr_variant_info *out) {
     cudaFuncAttributes a;
     GTR_CUDA_TRY(cudaFuncGetAttributes(&a, fn));

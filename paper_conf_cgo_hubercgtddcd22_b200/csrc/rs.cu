@@ -113,11 +113,26 @@ int gtr_internal_query_rs(gtr_ctx *ctx, const gtr_launch_cfg *cfg, gtr_variant_i
 
 namespace gtr {
 namespace rs {
+// Words 9..11 hold the pole's lookup-invariant factors of exp(12 i Z)
+// (Z = (E - EA)/2): |exp| = fast_exp(-12 Z.i) depends on EA.i only -- the
+// same operations as the lookup would do, so the same bits -- and the phase
+// factor exp(-6 i EA.r), which the lookup rotates by exp(6 i E).
 __global__ void k_wide_poles(const double *__restrict__ poles, int64_t n_rec, double *__restrict__ out) {
     for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n_rec * 12;
          i += (int64_t)gridDim.x * blockDim.x) {
         const int64_t r = i / 12, w = i - r * 12;
-        out[i] = w < 9 ? __ldg(poles + r * 9 + w) : 0.0;
+        double v;
+        if (w < 9) {
+            v = __ldg(poles + r * 9 + w);
+        } else if (w == 9) {
+            const double zi = (0.0 - __ldg(poles + r * 9 + 1)) * 0.5;     // Z.i, exact
+            v = fast_exp(-12.0 * zi);
+        } else {
+            double sp, cp;
+            sincos(6.0 * __ldg(poles + r * 9 + 0), &sp, &cp);
+            v = w == 10 ? cp : sp;
+        }
+        out[i] = v;
     }
 }
 }  // namespace rs

@@ -104,13 +104,13 @@ __device__ __forceinline__ cx fast_cexp(cx z) {
 __device__ __forceinline__ bool faddeeva_inner_branch(cx Z) {
     return __dadd_rn(__dmul_rn(Z.r, Z.r), __dmul_rn(Z.i, Z.i)) < 36.0;
 }
-__device__ __forceinline__ cx faddeeva_series(cx Z) {
+// e = exp(12 i Z) (fast_cexp); the wide-pole path passes it precomputed
+__device__ __forceinline__ cx faddeeva_series(cx Z, cx e) {
     {
         constexpr double an[10] = {2.758402e-01, 2.245740e-01, 1.594149e-01, 9.866577e-02, 5.324414e-02,
                                    2.505215e-02, 1.027747e-02, 3.676164e-03, 1.146494e-03, 3.117570e-04};
         constexpr double dl[10] = {9.869604e+00, 3.947842e+01, 8.882644e+01, 1.579137e+02, 2.467401e+02,
                                    3.553058e+02, 4.836106e+02, 6.316547e+02, 7.994379e+02, 9.869604e+02};
-        const cx e = fast_cexp(cx{-12.0 * Z.i, 12.0 * Z.r});          // exp(i 12 Z)
         const cx den = {12.0 * Z.r, 12.0 * Z.i};                        // 12 Z
         const double b_r = 144.0 * (Z.r * Z.r - Z.i * Z.i), b_i = 144.0 * (2.0 * Z.r * Z.i);   // 144 Z^2
         // batched inversion of q_0 = |12 Z|^2, q_{n+1} = |dl_n - 144 Z^2|^2
@@ -170,8 +170,25 @@ __device__ __forceinline__ cx faddeeva_series(cx Z) {
         return {W0.r - 8.124330e+01 * zs.i, W0.i + 8.124330e+01 * zs.r};   // W0 + i 81.2433 Z sum
     }
 }
+__device__ __forceinline__ cx faddeeva_asymptotic(cx Z);
 __device__ __forceinline__ cx faddeeva(cx Z) {
-    if (faddeeva_inner_branch(Z)) return faddeeva_series(Z);
+    if (faddeeva_inner_branch(Z)) return faddeeva_series(Z, fast_cexp(cx{-12.0 * Z.i, 12.0 * Z.r}));   // exp(i 12 Z)
+    return faddeeva_asymptotic(Z);
+}
+// the wide-pole form: exp(12 i Z) = t1 * exp(6 i E) * exp(-6 i EA.r), the
+// pole's factors t1 = fast_exp(-12 Z.i) (bit-identical to computing it here)
+// and (cos, sin)(6 EA.r) precomputed in its record, (cE, sE) = (cos, sin)(6 E)
+// once per lookup: one complex rotation instead of fast_exp + sincos per pole
+// (6 E - 6 EA.r = 12 Z.r in exact arithmetic; the phase differs from the
+// oracle's 12 Z.r by rounding only, ~1e-15 rad, within R-RS-tol)
+__device__ __forceinline__ cx faddeeva_pre(cx Z, double t1, double cp, double sp, double cE, double sE) {
+    if (faddeeva_inner_branch(Z)) {
+        const double c = cE * cp + sE * sp, sn = sE * cp - cE * sp;
+        return faddeeva_series(Z, cx{t1 * c, t1 * sn});
+    }
+    return faddeeva_asymptotic(Z);
+}
+__device__ __forceinline__ cx faddeeva_asymptotic(cx Z) {
     const cx a = {0.512424224754768462984202823134979415014943561548661637413182, 0.0};
     const cx b = {0.275255128608410950901357962647054304017026259671664935783653, 0.0};
     const cx c = {0.051765358792987823963876628425793170829107067780337219430904, 0.0};
@@ -191,7 +208,7 @@ struct TagSig {};
 
 // microscopic XS of nuclide nuc at energy E (4 channels) into micro
 template <class K, class LM>
-__device__ __forceinline__ void micro_xs(const Params &P, int64_t nuc, double E, LM &micro) {
+__device__ __forceinline__ void micro_xs(const Params &P, int64_t nuc, double E, double cE, double sE, LM &micro) {
     Local<K, double, 8, TagSigTF> sf;     // sigTfactors[4] complex
     Local<K, double, 2, TagZ> Zv;
     Local<K, double, 2, TagW> Wv;
@@ -235,11 +252,13 @@ __device__ __forceinline__ void micro_xs(const Params &P, int64_t nuc, double E,
     sig[1] = E * wA;
     sig[2] = E * wF;
     // one pole (c4 step 4), in pole order
-    auto pole = [&](double2 EA, double2 RT, double2 RA, double2 RF, int lv) {
+    // pre: a wide record's {t1, cos 6EA.r, sin 6EA.r}
+    auto pole = [&](double2 EA, double2 RT, double2 RA, double2 RF, int lv, bool pre, double t1, double cp,
+                    double sp) {
         const cx Z = cmul(csub(cx{E, 0.0}, cx{EA.x, EA.y}), cx{0.5, 0.0});
         Zv[0] = Z.r;
         Zv[1] = Z.i;
-        const cx W = faddeeva(cx{Zv[0], Zv[1]});
+        const cx W = pre ? faddeeva_pre(cx{Zv[0], Zv[1]}, t1, cp, sp, cE, sE) : faddeeva(cx{Zv[0], Zv[1]});
         Wv[0] = W.r;
         Wv[1] = W.i;
         const cx Wl = {Wv[0], Wv[1]};
@@ -271,18 +290,21 @@ __device__ __forceinline__ void micro_xs(const Params &P, int64_t nuc, double E,
             const double *pr = base + (int64_t)p * 12;
             const double2 EA = nEA, RT = nRT;
             double2 RA, RF;
+            double w8, t1, cp, sp;
             ld256(pr + 4, RA.x, RA.y, RF.x, RF.y);
-            const int lv = __ldg(reinterpret_cast<const int *>(pr + 8));
+            ld256(pr + 8, w8, t1, cp, sp);                       // l_value + the pole's exp factors
             if (p + 1 < se.y) ld256(pr + 12, nEA.x, nEA.y, nRT.x, nRT.y);
-            pole(EA, RT, RA, RF, lv);
+            pole(EA, RT, RA, RF, __double2loint(w8), true, t1, cp, sp);
         }
 #else
         for (int32_t p = se.x; p < se.y; p++) {
             const double *pr = base + (int64_t)p * 12;
             double2 EA, RT, RA, RF;
+            double w8, t1, cp, sp;
             ld256(pr + 0, EA.x, EA.y, RT.x, RT.y);
             ld256(pr + 4, RA.x, RA.y, RF.x, RF.y);
-            pole(EA, RT, RA, RF, __ldg(reinterpret_cast<const int *>(pr + 8)));
+            ld256(pr + 8, w8, t1, cp, sp);
+            pole(EA, RT, RA, RF, __double2loint(w8), true, t1, cp, sp);
         }
 #endif
     } else {
@@ -290,7 +312,7 @@ __device__ __forceinline__ void micro_xs(const Params &P, int64_t nuc, double E,
             const double *pr = P.poles + (nuc * P.max_poles + p) * 9;
             pole(make_double2(__ldg(pr + 0), __ldg(pr + 1)), make_double2(__ldg(pr + 2), __ldg(pr + 3)),
                  make_double2(__ldg(pr + 4), __ldg(pr + 5)), make_double2(__ldg(pr + 6), __ldg(pr + 7)),
-                 __ldg(reinterpret_cast<const int *>(pr + 8)));
+                 __ldg(reinterpret_cast<const int *>(pr + 8)), false, 0.0, 0.0, 0.0);
         }
     }
     micro[0] = sig[0];
@@ -309,11 +331,14 @@ __device__ __forceinline__ void lookup(const Params &P, uint64_t i, uint32_t *ta
     const int mat = smp::sample_material(seed[0]);
 #pragma unroll
     for (int c = 0; c < 4; c++) macro[c] = 0.0;
+    // the lookup's rotation exp(6 i E) for the wide records' precomputed pole factors
+    double sE = 0.0, cE = 1.0;
+    if (P.poles_wide) sincos(6.0 * E, &sE, &cE);
     const int nn = __ldg(P.num_nucs + mat);
     for (int j = 0; j < nn; j++) {
         const int64_t nuc = __ldg(P.mats + (int64_t)mat * P.max_num_nucs + j);
         const double conc = __ldg(P.concs + (int64_t)mat * P.max_num_nucs + j);
-        micro_xs<K>(P, nuc, E, micro);
+        micro_xs<K>(P, nuc, E, cE, sE, micro);
 #pragma unroll
         for (int c = 0; c < 4; c++) macro[c] += micro[c] * conc;
     }
@@ -369,13 +394,43 @@ template <class K> struct LookupRegion {
 #define GTR_RS_LPT 32   // measured (10M, SPMD / CSM): 8: 93.7 / 84.2, 16: 104.1 / 98.4, 32: 105.8 / 99.1 M lookups/s
 #endif
 constexpr uint32_t kBucketLookupsPerThread = GTR_RS_LPT;
+// Buckets are (material, energy bin): inside a material bucket the lookups
+// are also grouped by energy (GTR_RS_EBINS bins of [0,1)), so the 32 lanes
+// of a warp claim lookups of nearly equal energy -- they read the same
+// windows and pole records (one L1 request per warp instead of one per lane)
+// and run pole loops of equal length.  Results unchanged.
+#ifndef GTR_RS_BALANCED
+#define GTR_RS_BALANCED 0
+#endif
+#ifndef GTR_RS_EBINS
+#define GTR_RS_EBINS 64
+#endif
+constexpr int kEBins = GTR_RS_EBINS;
+constexpr int kBuckets = 12 * kEBins;
+__device__ __forceinline__ int bucket_of(int mat, double E) {
+    int eb = (int)(E * (double)kEBins);
+    eb = eb < kEBins - 1 ? eb : kEBins - 1;
+    return mat * kEBins + eb;
+}
 template <class K> struct ChunkBuf {
     static constexpr int CH = kBucketLookupsPerThread * K::NT;
     uint16_t perm[CH];
-    uint8_t mat[CH];
-    uint32_t cnt[12], cur[12];
+    uint16_t key[CH];                // bucket of lookup k
+    uint32_t cnt[kBuckets], cur[kBuckets];
     unsigned int next;
 };
+// sequential code of a chunk: zero the counters / turn them into bucket offsets
+template <class K> __device__ __forceinline__ void buckets_reset(ChunkBuf<K> &b) {
+    for (int m = 0; m < kBuckets; m++) b.cnt[m] = 0;
+    b.next = 0;
+}
+template <class K> __device__ __forceinline__ void buckets_offsets(ChunkBuf<K> &b) {
+    uint32_t off = 0;
+    for (int m = 0; m < kBuckets; m++) {
+        b.cur[m] = off;
+        off += b.cnt[m];
+    }
+}
 template <class K> __device__ __forceinline__ ChunkBuf<K> &chunk_buf() {
     if constexpr (K::MODE == NATIVE) return *reinterpret_cast<ChunkBuf<K> *>(g_dyn);   // no runtime state
     const uint32_t off = tstate_bytes<K>() + (uint32_t)K::BLOCK * g_ts.rp.sm_stride_words * 8u;
@@ -389,10 +444,11 @@ template <class K> struct SampleRegion {
         ChunkBuf<K> &b = chunk_buf<K>();
         for_static<K>(0, (int64_t)cnt, [&](int64_t k) {
             uint64_t s = smp::lcg_jump(g_p.seed, 2ULL * (base + (uint64_t)k));
-            (void)smp::lcg_uniform(s);                  // the energy draw
+            const double E = smp::lcg_uniform(s);       // the energy draw
             const int m = smp::sample_material(s);
-            b.mat[k] = (uint8_t)m;
-            atomicAdd(&b.cnt[m], 1u);
+            const int key = bucket_of(m, E);
+            b.key[k] = (uint16_t)key;
+            atomicAdd(&b.cnt[key], 1u);
         });
     }
 };
@@ -402,7 +458,7 @@ template <class K> struct ScatterRegion {
         const uint64_t cnt = static_cast<const Chunk *>(a)->count;
         ChunkBuf<K> &b = chunk_buf<K>();
         for_static<K>(0, (int64_t)cnt, [&](int64_t k) {
-            const uint32_t pos = atomicAdd(&b.cur[b.mat[k]], 1u);
+            const uint32_t pos = atomicAdd(&b.cur[b.key[k]], 1u);
             b.perm[pos] = (uint16_t)k;
         });
     }
@@ -459,18 +515,9 @@ template <class K> __global__ void __launch_bounds__(K::BLOCK, K::NT == 128 ? (K
             return;
         }
         ChunkBuf<K> &b = chunk_buf<K>();
-        guarded<K>([&] {
-            for (int m = 0; m < 12; m++) b.cnt[m] = 0;
-            b.next = 0;
-        });
+        guarded<K>([&] { buckets_reset(b); });
         parallel<K, SampleRegion<K>>(chunk.get());
-        guarded<K>([&] {
-            uint32_t off = 0;
-            for (int m = 0; m < 12; m++) {
-                b.cur[m] = off;
-                off += b.cnt[m];
-            }
-        });
+        guarded<K>([&] { buckets_offsets(b); });
         parallel<K, ScatterRegion<K>>(chunk.get());
         parallel<K, BucketRegion<K>>(chunk.get());
     });
@@ -497,19 +544,12 @@ __global__ void __launch_bounds__(K::NT, K::NT == 128 ? GTR_RS_MINB : 1) kernel_
         if (threadIdx.x == 0) {
             chunk.base = g_p.first + c * ch;
             chunk.count = (c * ch + ch <= n) ? ch : n - c * ch;
-            for (int m = 0; m < 12; m++) b.cnt[m] = 0;
-            b.next = 0;
+            buckets_reset(b);
         }
         __syncthreads();
         SampleRegion<K>::run(&chunk);
         __syncthreads();
-        if (threadIdx.x == 0) {
-            uint32_t off = 0;
-            for (int m = 0; m < 12; m++) {
-                b.cur[m] = off;
-                off += b.cnt[m];
-            }
-        }
+        if (threadIdx.x == 0) buckets_offsets(b);
         __syncthreads();
         ScatterRegion<K>::run(&chunk);
         __syncthreads();
@@ -542,8 +582,13 @@ template <class K> struct OpRt {
             GTR_CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, fn, K::BLOCK, L.dyn_smem));
             return fill_info<K>(fn, L, per_sm, a.info);
         }
+#if GTR_RS_BALANCED
+        a.P.chunk = balanced_chunk(a.P.n, (a.P.plain ? kLookupsPerThreadPerChunk : kBucketLookupsPerThread) * K::NT,
+                                   L.teams);
+#else
         a.P.chunk = fit_chunk(a.P.n, (a.P.plain ? kLookupsPerThreadPerChunk : kBucketLookupsPerThread) * K::NT,
                               L.teams);
+#endif
         kernel_rt<K><<<L.teams, L.block, L.dyn_smem, a.stream>>>(a.P, L.rp);
         GTR_CUDA_TRY(cudaGetLastError());
         return GTR_OK;

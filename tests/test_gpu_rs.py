@@ -97,13 +97,23 @@ def dev_narrow(rs):
     return RsDevice(rs[0], wide_poles=False)
 
 
-def test_rs_wide_poles_builder(dev, rs):
-    """poles_wide[r] = the 72-byte record's 9 words + 3 zero words."""
+def test_rs_wide_poles_builder(orc, dev, rs):
+    """poles_wide[r] = the 72-byte record's 9 words + the pole's lookup-
+    invariant factors of exp(12 i Z): word 9 = fast_exp(-12 Z.i) with Z.i =
+    -EA.i/2 -- bit-identical to the oracle's orc_fast_exp of the same
+    argument -- and words 10, 11 = cos, sin(6 EA.r) (CUDA libm vs numpy:
+    within 2 ulp)."""
     t = rs[0]
     raw = np.ascontiguousarray(t["poles"]).view(np.float64).reshape(-1, 9)
     got = dev.poles_wide.cpu().numpy()
     assert np.array_equal(got[:, :9].view(np.uint64), raw.view(np.uint64))
-    assert (got[:, 9:] == 0).all()
+    ea_r, ea_i = raw[:, 0], raw[:, 1]
+    idx = np.random.default_rng(0).integers(0, len(raw), 2000)
+    for r in idx:
+        zi = (0.0 - ea_i[r]) * 0.5
+        assert got[r, 9] == orc.fast_exp(-12.0 * zi)
+    np.testing.assert_allclose(got[:, 10], np.cos(6.0 * ea_r), rtol=0, atol=5e-16)
+    np.testing.assert_allclose(got[:, 11], np.sin(6.0 * ea_r), rtol=0, atol=5e-16)
 
 
 @pytest.mark.parametrize("cfg", [(0, 0, 0, 128), (2, 3, 1, 128), (3, 3, 1, 128), (3, 0, 0, 128), (4, 3, 1, 128),
