@@ -122,9 +122,7 @@ struct ThreadState {
     uint8_t nested;   // serialized nested parallel depth
     uint8_t level;    // SPMD: this thread's parallel level
     uint32_t gsp;     // global fallback stack top (words)
-    uint32_t bphase;  // F_BCAST_1BAR: broadcast slot of this thread's next guarded_bcast
-    uint32_t pad;
-};
+};                    // 8 bytes: a warp's accesses to .sp are 2-way bank conflicted at most
 // PL_COALESCED only: per-lane + per-warp allocation state (after ThreadState)
 struct CoalState {
     uint32_t igsp;    // this lane's own global stack top (divergent calls)
@@ -139,9 +137,16 @@ extern __shared__ __align__(16) uint8_t g_dyn[];
 template <class K> __host__ __device__ constexpr uint32_t coal_offset() {
     return (uint32_t)((K::BLOCK * sizeof(ThreadState) + 15) / 16 * 16);
 }
-template <class K> __host__ __device__ constexpr uint32_t tstate_bytes() {
+template <class K> __host__ __device__ constexpr uint32_t bphase_offset() {
     return coal_offset<K>() + (K::PL == 4 /*PL_COALESCED*/ ? (uint32_t)((K::BLOCK * sizeof(CoalState) + 15) / 16 * 16)
                                                            : 0u);
+}
+// F_BCAST_1BAR only: one u32 per thread, the slot of its next guarded_bcast
+template <class K> __host__ __device__ constexpr uint32_t tstate_bytes() {
+    return bphase_offset<K>() + ((K::FLAGS & 1 /*F_BCAST_1BAR*/) ? (uint32_t)((K::BLOCK * 4 + 15) / 16 * 16) : 0u);
+}
+template <class K> __device__ __forceinline__ uint32_t &bphase() {
+    return reinterpret_cast<uint32_t *>(g_dyn + bphase_offset<K>())[threadIdx.x];
 }
 template <class K> __device__ __forceinline__ CoalState &cstate() {
     return reinterpret_cast<CoalState *>(g_dyn + coal_offset<K>())[threadIdx.x];
@@ -294,13 +299,14 @@ enum class Role { Main, Worker, Exit };
 // code, guarded).
 template <class K> __device__ __forceinline__ Role team_init(const RtParams &rp) {
     if constexpr (K::TSTATE) {
-        ThreadState z = {0, 0, 0, 0, 0, 0};
+        ThreadState z = {0, 0, 0, 0};
         tstate<K>() = z;
     }
     if constexpr (K::PL == 4 /*PL_COALESCED*/) {
         CoalState c = {0, 0, 0, 0, 0, 0};
         cstate<K>() = c;
     }
+    if constexpr ((K::FLAGS & F_BCAST_1BAR) != 0) bphase<K>() = 0;
     if constexpr (K::GENERIC_LIKE) {
         if ((int)threadIdx.x >= K::NT) {
             if ((int)threadIdx.x != K::MAIN_HW) return Role::Exit;
@@ -469,8 +475,8 @@ template <class K, class T, class F> __device__ __forceinline__ T guarded_bcast(
     } else if constexpr (K::MODE == SPMD) {
         int b = 0;
         if constexpr ((K::FLAGS & F_BCAST_1BAR) != 0) {
-            b = (int)(tstate<K>().bphase & 1u);
-            tstate<K>().bphase ^= 1u;
+            b = (int)(bphase<K>() & 1u);
+            bphase<K>() ^= 1u;
         }
         if (threadIdx.x == 0) *reinterpret_cast<T *>(&g_ts.bcast[b]) = f();
         cta_sync<K>();
