@@ -18,7 +18,7 @@ template <int NT> __global__ void __launch_bounds__(NT) kernel_native(Params P) 
     if (P.req) { P.first = P.req->first; P.n = P.req->n; P.seed = P.req->seed; }
     __syncthreads();
     const uint64_t stride = (uint64_t)gridDim.x * NT;
-    if (P.s_perm) {                                   // sorted mode: thread per sorted position
+    if (P.s_rec) {                                    // sorted mode: thread per sorted position
         for (uint64_t q = (uint64_t)blockIdx.x * NT + threadIdx.x; q < P.n; q += stride)
             lookup_sorted<KN>(P, q, tally);
     } else if (P.history) {                           // history mode: thread per particle
@@ -52,15 +52,22 @@ __device__ __forceinline__ int64_t count_below(const double *__restrict__ a, int
     }
     return lo;
 }
-// position of energy (n,k) in the union = number of smaller energies
+// position of energy (n,k) in the union: the number of energies before it in
+// (energy, nuclide, gridpoint) order -- smaller energies, equal energies of
+// lower nuclides, and equal energies earlier in its own (sorted) nuclide, of
+// which there are k - #{smaller}: so its own nuclide contributes exactly k.
+// Distinct ranks even with duplicate energies (equal values in any order
+// make the same ascending egrid).
 __global__ void k_union_scatter(const double *__restrict__ e, int64_t n_iso, int64_t n_gp,
                                 double *__restrict__ egrid) {
     const int64_t total = n_iso * n_gp;
     for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < total;
          i += (int64_t)gridDim.x * blockDim.x) {
         const double x = e[i];
-        int64_t rank = 0;
-        for (int64_t m = 0; m < n_iso; m++) rank += count_below(e + m * n_gp, n_gp, x, false);
+        const int64_t n = i / n_gp, k = i - n * n_gp;
+        int64_t rank = k;
+        for (int64_t m = 0; m < n_iso; m++)
+            if (m != n) rank += count_below(e + m * n_gp, n_gp, x, m < n);
         egrid[rank] = x;
     }
 }
@@ -68,17 +75,17 @@ __global__ void k_fill_nan(double *p, int64_t n) {
     for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
         p[i] = __longlong_as_double(0x7FF8000000000000LL);
 }
-// strictly increasing (also catches unwritten NaN slots = duplicate ranks)
+// ascending (also catches unwritten NaN slots: unsorted nuclides or NaN input)
 __global__ void k_check_increasing(const double *__restrict__ eg, int64_t n, uint32_t *err) {
     for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n;
          i += (int64_t)gridDim.x * blockDim.x) {
         const double a = eg[i];
         bool ok = (a == a);
-        if (i + 1 < n) ok = ok && (eg[i + 1] > a);
-        if (!ok) atomicOr(err, (uint32_t)ERR_DUP_ENERGY);
+        if (i + 1 < n) ok = ok && (eg[i + 1] >= a);
+        if (!ok) atomicOr(err, (uint32_t)ERR_BUILD);
     }
 }
-// index[u][n] = clamp(#{k: e_n[k] <= egrid[u]} - 1, 0, n_gp - 2)
+// closed form cf(u) = clamp(#{k: e_n[k] <= egrid[u]} - 1, 0, n_gp - 2)
 __global__ void k_index_grid(const double *__restrict__ e, int64_t n_iso, int64_t n_gp,
                              const double *__restrict__ egrid, int64_t n_union, int32_t *__restrict__ idx) {
     const int64_t total = n_union * n_iso;
@@ -88,6 +95,52 @@ __global__ void k_index_grid(const double *__restrict__ e, int64_t n_iso, int64_
         int64_t c = count_below(e + n * n_gp, n_gp, __ldg(egrid + u), true) - 1;
         c = c < 0 ? 0 : (c > n_gp - 2 ? n_gp - 2 : c);
         idx[t] = (int32_t)c;
+    }
+}
+// XSBench's sequential rule (idx_low advances by at most one per
+// union point, idx(-1) = 0) from the closed form: the step is taken exactly
+// when cf(u) > idx(u-1) (e_n[idx+1] <= egrid[u] <=> cf(u) >= idx+1 for
+// idx < n_gp - 2), and idx(u) <= cf(u) throughout, so
+// idx(u) = min(idx(u-1) + 1, cf(u)) = u + min(1, min_{v<=u} (cf(v) - v)):
+// a prefix minimum down each column.  Without duplicate energies cf grows by
+// at most one per union point and idx = cf (the pass changes nothing).
+// Blocked scan: (1) per block of kIdxRows rows the column minimum of cf - u,
+// (2) per column the exclusive prefix minimum over blocks, (3) the rewrite.
+constexpr int64_t kIdxRows = 4096;
+__global__ void k_index_colmin(const int32_t *__restrict__ idx, int64_t n_union, int64_t n_iso,
+                               int32_t *__restrict__ bmin) {
+    const int64_t nblk = (n_union + kIdxRows - 1) / kIdxRows;
+    for (int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; t < nblk * n_iso;
+         t += (int64_t)gridDim.x * blockDim.x) {
+        const int64_t blk = t / n_iso, n = t - blk * n_iso;
+        const int64_t u1 = min(n_union, (blk + 1) * kIdxRows);
+        int32_t m = INT32_MAX;
+        for (int64_t u = blk * kIdxRows; u < u1; u++) m = min(m, (int32_t)(idx[u * n_iso + n] - u));
+        bmin[t] = m;
+    }
+}
+__global__ void k_index_colscan(int32_t *__restrict__ bmin, int64_t nblk, int64_t n_iso) {
+    for (int64_t n = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; n < n_iso; n += (int64_t)gridDim.x * blockDim.x) {
+        int32_t run = INT32_MAX;                      // exclusive: the minimum over earlier blocks
+        for (int64_t b = 0; b < nblk; b++) {
+            const int32_t v = bmin[b * n_iso + n];
+            bmin[b * n_iso + n] = run;
+            run = min(run, v);
+        }
+    }
+}
+__global__ void k_index_sequential(int32_t *__restrict__ idx, int64_t n_union, int64_t n_iso,
+                                   const int32_t *__restrict__ carry) {
+    const int64_t nblk = (n_union + kIdxRows - 1) / kIdxRows;
+    for (int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; t < nblk * n_iso;
+         t += (int64_t)gridDim.x * blockDim.x) {
+        const int64_t blk = t / n_iso, n = t - blk * n_iso;
+        const int64_t u1 = min(n_union, (blk + 1) * kIdxRows);
+        int32_t run = carry[t];
+        for (int64_t u = blk * kIdxRows; u < u1; u++) {
+            run = min(run, (int32_t)(idx[u * n_iso + n] - u));
+            idx[u * n_iso + n] = (int32_t)(u + min(1, run));
+        }
     }
 }
 
@@ -114,7 +167,7 @@ template <int NT> int run_native(LaunchArgs &a) {
 template <int NT> int run_native_bucketed(LaunchArgs &a) {
     using KN = Cfg<NATIVE, PL_STACK, true, NT>;
     const void *fn = reinterpret_cast<const void *>(&kernel_native_bucketed<KN>);
-    const uint32_t smem = (uint32_t)sizeof(ChunkBuf<KN>);
+    const uint32_t smem = (uint32_t)(sizeof(ChunkBuf<KN>) > sizeof(CoBuf<KN>) ? sizeof(ChunkBuf<KN>) : sizeof(CoBuf<KN>));
     GTR_CUDA_TRY(cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
     int per_sm = 0;
     GTR_CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, fn, NT, smem));
@@ -165,7 +218,10 @@ int gtr_internal_query_xs(gtr_ctx *ctx, const gtr_launch_cfg *cfg, gtr_variant_i
 }
 
 extern "C" uint64_t gtr_xs_build_workspace_bytes(int64_t n_iso, int64_t n_gp) {
-    return (uint64_t)n_iso * (uint64_t)n_gp * 8u;
+    // energies (8 B each) + the index builder's per-block column minima
+    const uint64_t total = (uint64_t)n_iso * (uint64_t)n_gp;
+    const uint64_t nblk = (total + (uint64_t)xs::kIdxRows - 1) / (uint64_t)xs::kIdxRows;
+    return total * 8u + nblk * (uint64_t)n_iso * 4u;
 }
 
 static int grid_blocks(gtr_ctx *ctx, int64_t work, int threads) {
@@ -199,6 +255,13 @@ extern "C" int gtr_xs_build_index_grid(gtr_ctx *ctx, const double *d_grid, int64
     xs::k_extract_energies<<<grid_blocks(ctx, total, 256), 256, 0, s>>>(d_grid, total, e);
     xs::k_index_grid<<<grid_blocks(ctx, total * n_iso, 256), 256, 0, s>>>(e, n_iso, n_gp, d_egrid, total,
                                                                           d_index_out);
+    // the sequential rule (differs from the closed form only where energies
+    // repeat); block minima live in the workspace after the energies
+    const int64_t nblk = (total + xs::kIdxRows - 1) / xs::kIdxRows;
+    int32_t *bmin = reinterpret_cast<int32_t *>(e + total);
+    xs::k_index_colmin<<<grid_blocks(ctx, nblk * n_iso, 256), 256, 0, s>>>(d_index_out, total, n_iso, bmin);
+    xs::k_index_colscan<<<grid_blocks(ctx, n_iso, 128), 128, 0, s>>>(bmin, nblk, n_iso);
+    xs::k_index_sequential<<<grid_blocks(ctx, nblk * n_iso, 256), 256, 0, s>>>(d_index_out, total, n_iso, bmin);
     GTR_CUDA_TRY(cudaGetLastError());
     return GTR_OK;
 }
@@ -306,37 +369,59 @@ extern "C" int gtr_xs_lookup_host(gtr_ctx *ctx, const gtr_launch_cfg *cfg, const
 
 // ---------------------------------------------------------------- sorted mode
 // XSBench's sorted event-based variant: sample every lookup,
-// counting-sort the lookups by (material, energy bucket), then run them in
+// sort the lookups by (material, unionized-grid index), then run them in
 // that order -- neighbouring threads share a material (equal-length nuclide
 // loops) and nearly equal energies (the same gridpoints, adjacent index-grid
-// rows).  Results are identical: each lookup's arithmetic is its own, the
-// tallies are sums.  Workspace (caller-owned, gtr_xs_sorted_workspace_bytes):
-//   key[n] u32 | mu[n] u32 (unsorted) | perm[n] u32 | smu[n] u32 | hist[12*NB] u32 | totals[256] u32
+// rows), which the warp-coherent nuclide loops (CoherentRegion) exploit.
+// Results are identical: each lookup's arithmetic is its own, the tallies
+// are sums.  The sort: counting sort by (material, u bucket) with 2^17
+// buckets per material, then each bucket (fuel: ~18 lookups) ordered by
+// (u, lookup) with a rank count -- a warp's 32 lookups then span ~50 union
+// points instead of a whole bucket.  Workspace (caller-owned,
+// gtr_xs_sorted_workspace_bytes), 16-byte aligned:
+//   rec0[n] SortRec | rec1[n] SortRec | key[n] u32 | hist[12*NB] u32 | totals u32
+// rec0 holds the samples in lookup order, then the final (ranked) order.
 namespace gtr {
 namespace xs {
-constexpr uint32_t kSortBuckets = 1u << 14;           // energy buckets per material
+constexpr uint32_t kSortBuckets = 1u << 17;           // u buckets per material
 constexpr uint32_t kSortBins = 12u * kSortBuckets;
+constexpr uint32_t kScanBlocks = kSortBins / 1024;
+constexpr uint32_t kRankMax = 256;                    // larger buckets keep the scatter's order
 
-__global__ void k_sort_sample(Params P, uint32_t *__restrict__ key, uint32_t *__restrict__ mu,
+__device__ __forceinline__ uint32_t sort_key(uint32_t mat, uint32_t u, int64_t n_union) {
+    uint32_t b = (uint32_t)(((uint64_t)u * kSortBuckets) / (uint64_t)n_union);
+    b = b < kSortBuckets ? b : kSortBuckets - 1;
+    return mat * kSortBuckets + b;
+}
+__device__ __forceinline__ void store_rec(SortRec *d, const SortRec &r) {
+    *reinterpret_cast<uint4 *>(d) =
+        make_uint4(r.k, r.mu, (uint32_t)__double2loint(r.E), (uint32_t)__double2hiint(r.E));
+}
+__global__ void k_sort_sample(Params P, SortRec *__restrict__ rec, uint32_t *__restrict__ key,
                               uint32_t *__restrict__ hist) {
     using KN = Cfg<NATIVE, PL_STACK, true, 128>;
+    const int64_t nu = P.grid_type == 0 ? P.n_union : (P.grid_type == 2 ? P.hash_bins : 1);
     for (uint64_t k = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; k < P.n;
          k += (uint64_t)gridDim.x * blockDim.x) {
         double E;
         int mat;
         int64_t u;
         sample<KN>(P, P.first + k, E, mat, u);
-        uint32_t eb = (uint32_t)(E * (double)kSortBuckets);
-        eb = eb < kSortBuckets ? eb : kSortBuckets - 1;
-        const uint32_t kk = (uint32_t)mat * kSortBuckets + eb;
+        // the nuclide grid has no u: bucket by energy (the same monotone role)
+        const uint32_t kk = P.grid_type == 1
+                                ? sort_key((uint32_t)mat, (uint32_t)(E * (double)kSortBuckets), (int64_t)kSortBuckets)
+                                : sort_key((uint32_t)mat, (uint32_t)u, nu);
         key[k] = kk;
-        mu[k] = ((uint32_t)mat << 28) | (uint32_t)u;
+        SortRec r;
+        r.k = (uint32_t)k;
+        r.mu = ((uint32_t)mat << 28) | (uint32_t)u;
+        r.E = E;
+        store_rec(rec + k, r);
         atomicAdd(hist + kk, 1u);
     }
 }
 // exclusive scan of hist[kSortBins] in place: per 1024-bin block a shared-
 // memory scan + the block total, then every block adds the totals before it
-constexpr uint32_t kScanBlocks = kSortBins / 1024;
 __global__ void __launch_bounds__(1024) k_sort_scan_local(uint32_t *hist, uint32_t *totals) {
     __shared__ uint32_t part[1024];
     uint32_t *h = hist + (size_t)blockIdx.x * 1024;
@@ -363,21 +448,40 @@ __global__ void __launch_bounds__(1024) k_sort_scan_add(uint32_t *hist, const ui
     __syncthreads();
     hist[(size_t)blockIdx.x * 1024 + threadIdx.x] += off;
 }
-__global__ void k_sort_scatter(uint64_t n, const uint32_t *__restrict__ key, const uint32_t *__restrict__ mu,
-                               uint32_t *__restrict__ cursor, uint32_t *__restrict__ perm,
-                               uint32_t *__restrict__ smu) {
+__global__ void k_sort_scatter(uint64_t n, const uint32_t *__restrict__ key, const SortRec *__restrict__ in,
+                               uint32_t *__restrict__ cursor, SortRec *__restrict__ out) {
     for (uint64_t k = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; k < n; k += (uint64_t)gridDim.x * blockDim.x) {
         const uint32_t pos = atomicAdd(cursor + key[k], 1u);
-        perm[pos] = (uint32_t)k;
-        smu[pos] = mu[k];
+        *reinterpret_cast<uint4 *>(out + pos) = __ldg(reinterpret_cast<const uint4 *>(in + k));
     }
 }
-static_assert(kSortBins % 1024 == 0 && kScanBlocks <= 256, "scan split");
+// order each bucket by (u, lookup): after the scatter cursor[b] is the end of
+// bucket b (= the start of b+1); position p moves to start + its rank
+__global__ void k_sort_rank(uint64_t n, const uint32_t *__restrict__ key, const uint32_t *__restrict__ end,
+                            const SortRec *__restrict__ in, SortRec *__restrict__ out) {
+    for (uint64_t p = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; p < n; p += (uint64_t)gridDim.x * blockDim.x) {
+        const uint4 v = __ldg(reinterpret_cast<const uint4 *>(in + p));
+        const uint32_t k = v.x, u = v.y & 0x0FFFFFFFu;
+        const uint32_t b = key[k];
+        const uint32_t s = b ? __ldg(end + b - 1) : 0u, e = __ldg(end + b);
+        uint32_t dest = (uint32_t)p;
+        if (e - s <= kRankMax) {
+            uint32_t r = 0;
+            for (uint32_t q = s; q < e; q++) {
+                const uint2 w = __ldg(reinterpret_cast<const uint2 *>(in + q));
+                const uint32_t uq = w.y & 0x0FFFFFFFu;
+                r += (uq < u || (uq == u && w.x < k)) ? 1u : 0u;
+            }
+            dest = s + r;
+        }
+        *reinterpret_cast<uint4 *>(out + dest) = v;
+    }
+}
 }  // namespace xs
 }  // namespace gtr
 
 extern "C" uint64_t gtr_xs_sorted_workspace_bytes(uint64_t n) {
-    return 16u * n + 4u * (uint64_t)(xs::kSortBins + 256);
+    return 36u * n + 4u * (uint64_t)(xs::kSortBins + xs::kScanBlocks);
 }
 
 extern "C" int gtr_xs_lookup_sorted(gtr_ctx *ctx, const gtr_launch_cfg *cfg, const gtr_xs_tables *tables,
@@ -387,21 +491,22 @@ extern "C" int gtr_xs_lookup_sorted(gtr_ctx *ctx, const gtr_launch_cfg *cfg, con
     if (!ctx || !cfg || !tables_ok(tables) || !d_out || !d_workspace) return GTR_EINVAL;
     if (n == 0) return GTR_OK;
     if (n > 0xFFFFFFFFull || workspace_bytes < gtr_xs_sorted_workspace_bytes(n) ||
-        (uint64_t)tables->n_union >= (1ull << 28) || (cfg->flags & GTR_F_HISTORY))
+        (reinterpret_cast<uintptr_t>(d_workspace) & 15u) || (uint64_t)tables->n_union >= (1ull << 28) ||
+        (cfg->flags & GTR_F_HISTORY))
         return GTR_EINVAL;
     if (!valid_cfg(cfg)) return GTR_EINVAL;
     cudaStream_t s = static_cast<cudaStream_t>(stream);
-    uint32_t *key = static_cast<uint32_t *>(d_workspace);
-    uint32_t *mu = key + n, *perm = key + 2 * n, *smu = key + 3 * n, *hist = key + 4 * n;
+    xs::SortRec *rec0 = static_cast<xs::SortRec *>(d_workspace), *rec1 = rec0 + n;
+    uint32_t *key = reinterpret_cast<uint32_t *>(rec1 + n), *hist = key + n;
     xs::Params P = xs::make_params(tables, first, n, seed, d_out, verify, nullptr);
     GTR_CUDA_TRY(cudaMemsetAsync(hist, 0, 4u * xs::kSortBins, s));
-    xs::k_sort_sample<<<grid_blocks(ctx, (int64_t)n, 256), 256, 0, s>>>(P, key, mu, hist);
+    xs::k_sort_sample<<<grid_blocks(ctx, (int64_t)n, 256), 256, 0, s>>>(P, rec0, key, hist);
     xs::k_sort_scan_local<<<xs::kScanBlocks, 1024, 0, s>>>(hist, hist + xs::kSortBins);
     xs::k_sort_scan_add<<<xs::kScanBlocks, 1024, 0, s>>>(hist, hist + xs::kSortBins);
-    xs::k_sort_scatter<<<grid_blocks(ctx, (int64_t)n, 256), 256, 0, s>>>(n, key, mu, hist, perm, smu);
+    xs::k_sort_scatter<<<grid_blocks(ctx, (int64_t)n, 256), 256, 0, s>>>(n, key, rec0, hist, rec1);
+    xs::k_sort_rank<<<grid_blocks(ctx, (int64_t)n, 256), 256, 0, s>>>(n, key, hist, rec1, rec0);
     GTR_CUDA_TRY(cudaGetLastError());
-    P.s_perm = perm;
-    P.s_mu = smu;
+    P.s_rec = rec0;
     xs::LaunchArgs a{ctx, cfg, P, s, nullptr};
     return xs::launch(a);
 }

@@ -21,7 +21,7 @@ _lib = C.CDLL(LIB_PATH)
 GTR_OK, GTR_EINVAL, GTR_ECUDA, GTR_ENOMEM, GTR_EHEAP, GTR_EDEVICE, GTR_EUNSUPPORTED = 0, -1, -2, -3, -4, -5, -6
 GENERIC, GENERIC_CASCADE, CSM, SPMD, NATIVE = 0, 1, 2, 3, 4
 PL_RUNTIME, PL_GLOBAL, PL_SHARED_STATIC, PL_STACK, PL_COALESCED = 0, 1, 2, 3, 4
-F_BCAST_1BAR, F_SEPARATE_GUARDS, F_PLAIN, F_HISTORY, F_TMA, F_NATIVE_BUCKETED = 1, 2, 4, 8, 16, 32
+F_BCAST_1BAR, F_SEPARATE_GUARDS, F_PLAIN, F_HISTORY, F_TMA, F_NATIVE_BUCKETED, F_SORTED = 1, 2, 4, 8, 16, 32, 64
 K_XS, K_SU3, K_RS, K_FORKJOIN, K_SEMANTICS, K_BARRIER_FLOOR = 0, 1, 2, 3, 4, 5
 MODE_NAMES = {GENERIC: "generic", GENERIC_CASCADE: "cascade", CSM: "csm", SPMD: "spmd", NATIVE: "native"}
 PL_NAMES = {PL_RUNTIME: "runtime", PL_GLOBAL: "global", PL_SHARED_STATIC: "shared_static", PL_STACK: "stack",

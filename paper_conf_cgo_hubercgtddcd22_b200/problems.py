@@ -53,7 +53,7 @@ class XsDevice:
             self.union_bins_log2 = int(union_bins_log2)
             self.union_bins = torch.empty((1 << self.union_bins_log2) + 1, dtype=torch.int32, device=device)
             G.gtr_xs_build_union_bins(ctx, self.egrid, self.n_union, self.union_bins_log2, self.union_bins, stream)
-        G.gtr_ctx_check(ctx, stream)           # duplicate energies -> GtrError
+        G.gtr_ctx_check(ctx, stream)           # unsorted or NaN energies -> GtrError
         p = lambda x: x.data_ptr() if x is not None else None   # noqa: E731
         self.tables = G.gtr_xs_tables(self.n_iso, self.n_gp, self.n_union, self.max_num_nucs,
                                       p(self.egrid), p(self.index_grid), self.grid.data_ptr(),

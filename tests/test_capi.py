@@ -27,7 +27,11 @@ def test_host_only_calls():
     from paper_conf_cgo_hubercgtddcd22_b200 import gtr
     assert gtr.gtr_version() == 1000
     assert "heap" in gtr.gtr_strerror(gtr.GTR_EHEAP)
-    assert gtr.gtr_xs_build_workspace_bytes(355, 11303) == 355 * 11303 * 8
+    # energies + one i32 column minimum per (4096 union points, nuclide)
+    total = 355 * 11303
+    assert gtr.gtr_xs_build_workspace_bytes(355, 11303) == total * 8 + -(-total // 4096) * 355 * 4
+    # sorted mode: two 16-byte records + a key per lookup, 12 x 2^17 bins + block totals
+    assert gtr.gtr_xs_sorted_workspace_bytes(17_000_000) == 36 * 17_000_000 + 4 * (12 * 2**17 + 12 * 2**17 // 1024)
 
 
 def test_library_is_sm100a():

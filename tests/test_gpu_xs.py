@@ -258,11 +258,54 @@ def test_invalid_configs_rejected(G, ctx, dev_small):
             G.gtr_xs_lookup(ctx, bad, dev_small.tables, 0, 10, X.SEED_L, out)
 
 
-def test_duplicate_energies_detected(G, ctx):
+def test_duplicate_energies_golden(G, ctx):
+    """The hand-worked duplicate-energy case (tests/golden/xs_dup_index.txt,
+    SURVEY c2.5): union grid and the sequential rule's lagging index grid."""
+    import os
+    from paper_conf_cgo_hubercgtddcd22_b200.problems import XsDevice
+    t = X.make_tables(2, 4)
+    t["grid"][0, :, 0] = [0.1, 0.2, 0.2, 0.5]
+    t["grid"][1, :, 0] = [0.2, 0.3, 0.6, 0.7]
+    golden = np.loadtxt(os.path.join(os.path.dirname(__file__), "golden", "xs_dup_index.txt"), dtype=np.int64)
+    dev = XsDevice(ctx, t, union_bins_log2=None)
+    assert np.array_equal(dev.egrid.cpu().numpy(), [0.1, 0.2, 0.2, 0.2, 0.3, 0.5, 0.6, 0.7])
+    assert np.array_equal(dev.index_grid.cpu().numpy(), golden)
+
+
+def test_duplicate_energies_sequential_rule(G, ctx, orc):
+    """Duplicate gridpoint energies within and across nuclides: the GPU
+    builders reproduce the oracle's union grid and its sequential-rule index
+    grid (which lags the closed-form count), and every mode's lookups match."""
     from paper_conf_cgo_hubercgtddcd22_b200.problems import XsDevice
     t = X.make_tables(3, 50)
-    t["grid"][1, 10, 0] = t["grid"][0, 20, 0]
-    t["grid"][1] = t["grid"][1][np.argsort(t["grid"][1, :, 0], kind="stable")]
+    g = t["grid"]
+    g[0, 11, 0] = g[0, 10, 0]                         # a pair within nuclide 0
+    g[2, 21, 0] = g[2, 22, 0] = g[2, 20, 0]           # a triple within nuclide 2
+    g[1, 30, 0] = g[0, 30, 0]                         # across nuclides
+    g[2, 40, 0] = g[0, 40, 0] = g[1, 40, 0]
+    for n in range(3):
+        g[n] = g[n][np.argsort(g[n, :, 0], kind="stable")]
+    P = orc.XsProblem(t)
+    closed = np.clip(np.stack([np.searchsorted(g[n, :, 0], P.egrid, side="right") - 1 for n in range(3)], 1),
+                     0, g.shape[1] - 2)
+    assert (P.index_grid != closed).any()             # the lag is exercised
+    for log2b in (None, 8):
+        dev = XsDevice(ctx, t, union_bins_log2=log2b)
+        assert np.array_equal(dev.egrid.cpu().numpy(), P.egrid)
+        assert np.array_equal(dev.index_grid.cpu().numpy(), P.index_grid)
+        n = 20000
+        o_out, o_v = P.run(0, n, X.SEED_L, 4, verify=True)
+        for c in (G.cfg(G.SPMD, G.PL_STACK, 1, 256), G.cfg(G.CSM, G.PL_STACK, 1, 128),
+                  G.cfg(G.GENERIC, G.PL_RUNTIME, 0, 128), G.cfg(G.NATIVE, G.PL_STACK, 1, 256),
+                  G.cfg(G.SPMD, G.PL_STACK, 1, 256, flags=G.F_PLAIN)):
+            _assert_same(*_run(G, ctx, dev, c, 0, n), o_out, o_v)
+        _assert_same(*_run_sorted(G, ctx, dev, G.cfg(G.SPMD, G.PL_STACK, 1, 256), 0, n), o_out, o_v)
+
+
+def test_unsorted_energies_detected(G, ctx):
+    from paper_conf_cgo_hubercgtddcd22_b200.problems import XsDevice
+    t = X.make_tables(3, 50)
+    t["grid"][1, 10, 0], t["grid"][1, 11, 0] = t["grid"][1, 11, 0], t["grid"][1, 10, 0]
     with pytest.raises(G.GtrError):
         XsDevice(ctx, t)
 
@@ -353,6 +396,34 @@ def test_sorted_mode_grid_types(G, ctx, dev_grid, small):
     assert np.array_equal(v["macro"].view(np.uint64), o_v["macro"].view(np.uint64))
 
 
+@pytest.fixture(scope="module")
+def dense(G, ctx, orc):
+    """68 nuclides x 2000 gridpoints and 300,000 lookups: after the sort a
+    warp's 32 lookups mostly share each nuclide's gridpoint pair, so the
+    warp-coherent path (CoherentRegion) takes its uniform branch for most
+    positions, its two-record branch for the rest and, near the sparse
+    materials, the direct gather of a k beyond the staged records."""
+    from paper_conf_cgo_hubercgtddcd22_b200.problems import XsDevice
+    t = X.make_tables(68, 2000)
+    P = orc.XsProblem(t)
+    return P, XsDevice(ctx, t)
+
+
+@pytest.mark.parametrize("cfg", [(3, 3, 1, 256, 0, 0), (3, 0, 0, 256, 0, 0), (3, 3, 1, 128, 3, 0),
+                                 (2, 3, 1, 256, 0, 0), (2, 1, 0, 128, 2, 0), (0, 3, 1, 256, 0, 0),
+                                 (1, 0, 0, 128, 0, 0), (3, 4, 0, 256, 0, 0), (4, 3, 1, 256, 0, 1),
+                                 (4, 3, 1, 128, 5, 1)],
+                         ids=lambda c: f"m{c[0]}_p{c[1]}_f{c[2]}_t{c[3]}_teams{c[4]}_nb{c[5]}")
+@pytest.mark.parametrize("first,n", [(0, 300000), (12345, 77777)])
+def test_sorted_coherent_dense(G, ctx, dense, cfg, first, n):
+    P, dev = dense
+    m, p, f, nt, teams, nb = cfg
+    o_out, o_v = P.run(first, n, X.SEED_L, 8, verify=True)
+    c = G.cfg(m, p, f, nt, num_teams=teams, flags=G.F_NATIVE_BUCKETED if nb else 0)
+    out, v = _run_sorted(G, ctx, dev, c, first, n)
+    _assert_same(out, v, o_out, o_v)
+
+
 def test_sorted_mode_rejects_small_workspace(G, ctx, dev_small):
     out = torch.zeros(18, dtype=torch.uint64, device="cuda")
     ws = torch.empty(1024, dtype=torch.uint8, device="cuda")
@@ -434,6 +505,14 @@ def test_large_config_bench_launch(G, ctx, orc):
         G.gtr_xs_lookup(ctx, G.cfg(mode, G.PL_STACK, 1, 256), dev.tables, 0, n, X.SEED_L, out)
         G.gtr_ctx_check(ctx)
         assert np.array_equal(out.cpu().numpy(), o_out), mode
+    # the sorted event mode (global counting sort + warp-coherent nuclide loops)
+    ws = torch.empty(G.gtr_xs_sorted_workspace_bytes(n), dtype=torch.uint8, device="cuda")
+    for mode in (G.SPMD, G.CSM):
+        out = torch.zeros(18, dtype=torch.uint64, device="cuda")
+        G.gtr_xs_lookup_sorted(ctx, G.cfg(mode, G.PL_STACK, 1, 256), dev.tables, 0, n, X.SEED_L, out, ws)
+        G.gtr_ctx_check(ctx)
+        assert np.array_equal(out.cpu().numpy(), o_out), ("sorted", mode)
+    del ws
     first, m = 9_876_543, 20000
     o2, ov = P.run(first, m, X.SEED_L, 8, verify=True)
     out, v = _run(G, ctx, dev, G.cfg(G.SPMD, G.PL_STACK, 1, 256), first, m)

@@ -76,7 +76,9 @@ for v in a.variants:
         e1.record()
         torch.cuda.synchronize()
         ms = e0.elapsed_time(e1) / a.reps
-        info = G.gtr_query_variant(G.K_XS, c)
+        qc = G.gtr_launch_cfg(c.num_teams, c.thread_limit, c.mode, c.placement, c.fold, c.smem_stack_bytes,
+                              c.flags | (G.F_SORTED if v.endswith("_sorted") else 0))
+        info = G.gtr_query_variant(G.K_XS, qc)
         print(f"{v:16s} {ms:8.3f} ms  {a.n / ms / 1e3:8.1f} M lookups/s  regs {info['regs']} "
               f"teams/SM {info['teams_per_sm']}  hash {int(out.cpu()[0])}", flush=True)
     G.gtr_ctx_check(ctx)
