@@ -33,6 +33,7 @@ N_ISO, N_GP, LOOKUPS_PER_GPU = 355, 11303, 17_000_000
 METRIC = "XSBench lookups/s per mode + fork/join ns; % HBM roofline at 1/2/4/8 B200"
 WORKLOAD = "XSBench large: 355 nuclides x 11,303 gridpoints, 17M lookups per GPU"
 BYTES_PER_NUCLIDE = 100     # 4 B index-grid entry + 2 x 48 B gridpoints
+FLOPS_PER_NUCLIDE = 28      # fp64 ops of one nuclide visit (c3.2), a division counted once
 
 
 def parse():
@@ -43,6 +44,9 @@ def parse():
     ap.add_argument("--impl", default="gtr", choices=["gtr", "reference"])
     ap.add_argument("--no-sweep", action="store_true", help="skip the per-mode / fork-join sweeps")
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--schedule", default="sorted", choices=["sorted", "bucketed"],
+                    help="headline schedule: XSBench's sorted event mode (sampling pass + sort by (material, "
+                         "grid index) + warp-coherent lookups) or the per-chunk bucketed schedule")
     ap.add_argument("--combine", default="auto", choices=["auto", "fused", "nccl"],
                     help="N > 1: combine of the 18 u64 results -- fused into the lookup kernel's epilogue over "
                          "peer memory (auto: if every rank set it up and it matches NCCL once), or NCCL all_reduce")
@@ -287,6 +291,28 @@ def run_gtr(a):
     head = G.cfg(G.SPMD, G.PL_STACK, 1, 256)
     out = torch.zeros(18, dtype=torch.uint64, device=dev)
     num_nucs = tables["num_nucs"].astype(np.int64)
+    sorted_ = a.schedule == "sorted"
+    wsp = torch.empty(G.gtr_xs_sorted_workspace_bytes(n), dtype=torch.uint8, device=dev) if sorted_ else None
+
+    def launch(ptrs, kev=None):
+        """One step's launches: (sort, then) the lookups into `out` or, with
+        peer pointers, into every rank's buffer (fused combine)."""
+        if kev is not None:
+            kev[0].record(stream)
+        if sorted_:
+            G.gtr_xs_sort_lookups(ctx, xs.tables, first, n, seed, wsp, stream)
+        if kev is not None:
+            kev[1].record(stream)
+        if sorted_ and ptrs is not None:
+            G.gtr_xs_lookup_presorted_peers(ctx, head, xs.tables, first, n, ptrs, wsp, stream)
+        elif sorted_:
+            G.gtr_xs_lookup_presorted(ctx, head, xs.tables, first, n, out, wsp, None, stream)
+        elif ptrs is not None:
+            G.gtr_xs_lookup_peers(ctx, head, xs.tables, first, n, seed, ptrs, stream)
+        else:
+            G.gtr_xs_lookup(ctx, head, xs.tables, first, n, seed, out, None, stream)
+        if kev is not None:
+            kev[2].record(stream)
 
     # N > 1: the 18-u64 combine is fused into the lookup kernel's epilogue
     # (teams add into every rank's buffer over NVLink peer memory, then one
@@ -307,11 +333,11 @@ def run_gtr(a):
     def step():
         nonlocal out
         if pc is not None:
-            G.gtr_xs_lookup_peers(ctx, head, xs.tables, first, n, seed, pc.ptrs(), stream)
+            launch(pc.ptrs())
             out = pc.finish()
             return
         out.zero_()
-        G.gtr_xs_lookup(ctx, head, xs.tables, first, n, seed, out, None, stream)
+        launch(None)
         if dist is not None:
             combine_results(out)
 
@@ -323,7 +349,10 @@ def run_gtr(a):
         # GTR_BENCH_DIST=1): the fused result against the NCCL all-reduce of
         # this rank's own lookups; all ranks switch to NCCL together if any differs
         loc = torch.zeros(18, dtype=torch.uint64, device=dev)
-        G.gtr_xs_lookup(ctx, head, xs.tables, first, n, seed, loc, None, stream)
+        if sorted_:
+            G.gtr_xs_lookup_sorted(ctx, head, xs.tables, first, n, seed, loc, wsp, None, stream)
+        else:
+            G.gtr_xs_lookup(ctx, head, xs.tables, first, n, seed, loc, None, stream)
         combine_results(loc)
         nccl_res = loc.cpu().numpy()
         fused_res = out.cpu().numpy() if pc is not None else None
@@ -340,7 +369,7 @@ def run_gtr(a):
 
     # timed region: K steps, barrier + sync on both sides, CUDA events on the
     # launching stream; per-launch kernel events for the roofline
-    kev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(a.steps)]
+    kev = [tuple(torch.cuda.Event(enable_timing=True) for _ in range(3)) for _ in range(a.steps)]
     e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     with Clocks(local) as clk:
         if dist is not None:
@@ -349,16 +378,11 @@ def run_gtr(a):
         e0.record(stream)
         for s in range(a.steps):
             if pc is not None:
-                ptrs = pc.ptrs()
-                kev[s][0].record(stream)
-                G.gtr_xs_lookup_peers(ctx, head, xs.tables, first, n, seed, ptrs, stream)
-                kev[s][1].record(stream)
+                launch(pc.ptrs(), kev[s])
                 out = pc.finish()
                 continue
             out.zero_()
-            kev[s][0].record(stream)
-            G.gtr_xs_lookup(ctx, head, xs.tables, first, n, seed, out, None, stream)
-            kev[s][1].record(stream)
+            launch(None, kev[s])
             if dist is not None:
                 combine_results(out)
         e1.record(stream)
@@ -367,44 +391,99 @@ def run_gtr(a):
             dist.barrier()
     G.gtr_ctx_check(ctx, stream)
     ms = e0.elapsed_time(e1) / a.steps
-    k_ms = float(np.mean([b.elapsed_time(c) for b, c in kev]))
+    k_ms = float(np.mean([b.elapsed_time(c) for _, b, c in kev]))        # the lookup kernel
+    sort_ms = float(np.mean([a0.elapsed_time(b) for a0, b, _ in kev]))   # sampling pass + sort
     res = out.cpu().numpy().astype(np.uint64)
-    t_ms = torch.tensor([ms, k_ms], dtype=torch.float64, device=dev)
+    t_ms = torch.tensor([ms, k_ms, sort_ms], dtype=torch.float64, device=dev)
     if dist is not None:
         max_over_ranks(t_ms)
-    ms, k_ms = float(t_ms[0]), float(t_ms[1])
+    ms, k_ms, sort_ms = float(t_ms[0]), float(t_ms[1]), float(t_ms[2])
     value = ws * n / (ms * 1e-3)
 
-    # algorithmic bytes of one launch (this rank): sum over sampled materials
-    # of num_nucs x 100 B; the material tallies of all ranks are in `res`
+    # algorithmic work of one step (this rank): the material tallies of all
+    # ranks are in `res`; per nuclide visit 100 B and 28 fp64
+    # flops (c3.2: f = (hi.e - E) / (hi.e - lo.e) 3, five channels x 3, five
+    # x (mul, add) into macro; a division counted as one flop)
     mat_tally = res[1:13].astype(np.int64)
-    alg_bytes_all = float((mat_tally * num_nucs).sum() * BYTES_PER_NUCLIDE)
-    alg_bytes = alg_bytes_all / ws
+    visits = float((mat_tally * num_nucs).sum()) / ws
+    alg_bytes = visits * BYTES_PER_NUCLIDE
     hbm, peak_kind = peaks()
-    achieved = alg_bytes / (k_ms * 1e-3) / 1e9
-    traffic, traffic_src = None, None
     import glob
-    profs = sorted(glob.glob(os.path.join(ROOT, "profiles", "r*_xs_headline_ncu.json")))
-    if profs:   # dram read+write bytes of the headline kernel from the latest `ncu --set full` capture
-        ks = [k for k in json.load(open(profs[-1]))["kernels"] if "Cfg<3, 3, 1, 256" in k["kernel"]]
-        if ks:
-            traffic, traffic_src = ks[0]["dram_bytes_per_launch"], os.path.relpath(profs[-1], ROOT)
+
+    def ncu_traffic(pattern, kname):
+        """dram read+write bytes per launch of `kname` from the latest `ncu --set full` capture"""
+        profs = sorted(glob.glob(os.path.join(ROOT, "profiles", pattern)))
+        if profs:
+            ks = [k for k in json.load(open(profs[-1]))["kernels"] if kname in k["kernel"]]
+            if ks:
+                return ks[0]["dram_bytes_per_launch"], os.path.relpath(profs[-1], ROOT)
+        return None, None
+    hbm_src = f"{peak_kind} MEASURED_PEAKS.json hbm_gbs" if peak_kind == "measured" \
+        else "fallback B200_PROFILING.md 6.65 TB/s"
+    if sorted_:
+        # the sorted lookups share each gridpoint pair across a warp: DRAM
+        # traffic is a few GB per launch, far below the 100 B per visit the
+        # gather model counts, and the kernel's busiest unit is the fp64 pipe
+        fp64 = fp64_peak(G, torch, ctx, stream)
+        fp64_src = ("measured: gtr_fp64_probe (independent DFMA chains, 2 flops each); nominal 148 SM x 64 fp64 "
+                    "lanes x 2 x 1.965 GHz = 37.2 TFLOP/s")
+        flops = visits * FLOPS_PER_NUCLIDE
+        achieved = flops / (k_ms * 1e-3) / 1e12
+        traffic, traffic_src = ncu_traffic("r*_xs_sorted_ncu.json", "kernel_rt_sorted<Cfg<3, 3, 1, 256")
+        roofline = {"bound": "alu", "achieved": achieved, "peak": fp64, "unit": "TFLOP/s",
+                    "frac": achieved / fp64, "traffic": traffic, "traffic_source": traffic_src,
+                    "kernel": "kernel_rt_sorted<SPMD, heap-to-stack, fold, 256> (the lookups in sorted order)",
+                    "kernel_ms": k_ms, "sort_ms": sort_ms, "alg_flops_per_launch": flops,
+                    "peak_source": fp64_src,
+                    "gather_model": {"alg_bytes_per_launch": alg_bytes, "unit": "GB/s",
+                                     "achieved_kernel": alg_bytes / (k_ms * 1e-3) / 1e9,
+                                     "achieved_step": alg_bytes / (ms * 1e-3) / 1e9, "hbm_peak": hbm,
+                                     "note": "SURVEY 8(d)'s 100 B per nuclide visit over the lookup kernel / "
+                                             "the whole step (sort included): above the HBM peak because a warp "
+                                             "reads each shared gridpoint pair once, not once per lookup"}}
+    else:
+        achieved = alg_bytes / (k_ms * 1e-3) / 1e9
+        traffic, traffic_src = ncu_traffic("r*_xs_headline_ncu.json", "Cfg<3, 3, 1, 256")
+        roofline = {"bound": "hbm", "achieved": achieved, "peak": hbm, "unit": "GB/s",
+                    "frac": achieved / hbm, "traffic": traffic, "traffic_source": traffic_src,
+                    "kernel_ms": k_ms, "alg_bytes_per_launch": alg_bytes, "peak_source": hbm_src}
 
     extra = {}
     if not a.no_sweep:      # 180 GB HBM: the XS tables stay resident
         extra["sharded"] = sharded_apps(G, torch, ctx, rank, ws, dist, stream, dev)
+    if rank == 0:
+        # the other schedule of the same step, outside the timed region: the
+        # bucketed kernel's HBM roofline (the gather model of SURVEY 8(d))
+        if sorted_:
+            def fb():
+                out.zero_()
+                G.gtr_xs_lookup(ctx, head, xs.tables, first, n, seed, out, None, stream)
+            bms = _time(torch, stream, fb, 5)
+            btr, bsrc = ncu_traffic("r*_xs_headline_ncu.json", "Cfg<3, 3, 1, 256")
+            extra["bucketed_schedule"] = {
+                "lookups_per_s": n / (bms * 1e-3), "ms": bms, "same_result": bool(np.array_equal(out.cpu().numpy(), res))
+                if ws == 1 else None,
+                "roofline": {"bound": "hbm", "achieved": alg_bytes / (bms * 1e-3) / 1e9, "peak": hbm, "unit": "GB/s",
+                             "frac": alg_bytes / (bms * 1e-3) / 1e9 / hbm, "traffic": btr, "traffic_source": bsrc,
+                             "peak_source": hbm_src}}
     if rank == 0 and not a.no_sweep:
         extra.update(sweeps(G, torch, ctx, xs, first, seed, stream, cpu=(ws == 1 and not a.no_cpu_baseline)))
 
     # e2e through the public host-buffer entry point (H2D request, D2H results)
     h_out = torch.zeros(18, dtype=torch.uint64).pin_memory()
     req = G.gtr_xs_request(first, n, seed)
-    G.gtr_xs_lookup_host(ctx, head, xs.tables, req, h_out, stream)
+
+    def e2e_call():
+        if sorted_:
+            G.gtr_xs_lookup_sorted_host(ctx, head, xs.tables, req, h_out, wsp, stream)
+        else:
+            G.gtr_xs_lookup_host(ctx, head, xs.tables, req, h_out, stream)
+    e2e_call()
     if dist is not None:
         dist.barrier()
     t0 = time.perf_counter()
     for _ in range(a.steps):
-        G.gtr_xs_lookup_host(ctx, head, xs.tables, req, h_out, stream)
+        e2e_call()
     e2e_s = (time.perf_counter() - t0) / a.steps
     t_e = torch.tensor([e2e_s], dtype=torch.float64, device=dev)
     if dist is not None:
@@ -417,32 +496,36 @@ def run_gtr(a):
         m = 2_000_000
         cpu, o_out = cpu_baseline(tables, first, m, seed)
         chk = torch.zeros(18, dtype=torch.uint64, device=dev)
-        G.gtr_xs_lookup(ctx, head, xs.tables, first, m, seed, chk, None, stream)
+        if sorted_:
+            G.gtr_xs_lookup_sorted(ctx, head, xs.tables, first, m, seed, chk, wsp, None, stream)
+        else:
+            G.gtr_xs_lookup(ctx, head, xs.tables, first, m, seed, chk, None, stream)
         parity = bool(np.array_equal(chk.cpu().numpy(), o_out))
         cpu.pop("seconds")
 
     if rank == 0:
+        variant = ("SPMD + heap-to-stack + folding, thread_limit 256; sorted event mode: sampling pass + sort by "
+                   "(material, grid index) + warp-coherent lookups, all inside the timed step") if sorted_ else \
+            "SPMD + heap-to-stack + folding, thread_limit 256; per-chunk (material, energy) bucketed schedule"
         line = {
             "metric": METRIC, "value": value, "unit": "lookups/s", "n_gpus": ws, "steps": a.steps,
             "warmup": a.warmup, "ms_per_step": ms, "higher_is_better": True, "scaling": "weak",
             "vs_baseline": None, "dtype": "f64", "data": "synthetic",
-            "config": {"workload": WORKLOAD, "variant": "SPMD + heap-to-stack + folding, thread_limit 256",
+            "config": {"workload": WORKLOAD, "variant": variant, "schedule": a.schedule,
                        "lookups_per_gpu": n, "parallelism": f"dp{ws}: lookups sharded over {ws} GPU(s)",
                        "combine": combine, "nranks": nranks, "combine_check": combine_check,
                        "l2": "no flush: inputs 5.9 GB per GPU >> 126 MB L2 (index grid 5.7 GB)",
                        "table_setup_s": round(t_setup, 2)},
             "hash": int(res[0]), "hash_mod_999983": int(res[0] % 999983),
-            "roofline": {"bound": "hbm", "achieved": achieved, "peak": hbm, "unit": "GB/s",
-                         "frac": achieved / hbm, "traffic": traffic, "traffic_source": traffic_src,
-                         "kernel_ms": k_ms, "alg_bytes_per_launch": alg_bytes,
-                         "peak_source": f"{peak_kind} MEASURED_PEAKS.json hbm_gbs" if peak_kind == "measured"
-                         else "fallback B200_PROFILING.md 6.65 TB/s"},
+            "roofline": roofline,
             "cpu_baseline": cpu, "parity_vs_oracle_2M_sample": parity,
             "e2e": {"value": ws * n / e2e_s, "unit": "lookups/s",
                     "h2d_bytes_per_step": 24, "d2h_bytes_per_step": 144,
-                    "note": "gtr_xs_lookup_host: pinned host request -> device, lookups, 18 u64 -> pinned host, "
+                    "note": ("gtr_xs_lookup_sorted_host" if sorted_ else "gtr_xs_lookup_host") +
+                            ": pinned host request -> device, lookups, 18 u64 -> pinned host, "
                             "stream sync; tables resident (uploaded once, table_setup_s)"},
-            "gpu_launches": a.steps,
+            # our kernels per step: sampling, 2 scan, scatter, rank, lookups (sorted); the lookups (bucketed)
+            "gpu_launches": a.steps * (6 if sorted_ else 1),
             "clocks": clk.summary(),
             "host": host_info(),
         }

@@ -17,8 +17,8 @@ __device__ __forceinline__ double lcg_uniform(uint64_t &s) {
     s = lcg_step(s);
     return __ull2double_rn(s) * 0x1p-63;     // exact scaling by 2^-63
 }
-// Jump ahead n steps: compose the affine map x -> a x + c by squaring.
-__device__ __forceinline__ uint64_t lcg_jump(uint64_t seed, uint64_t n) {
+// The affine map of n steps, x -> A x + C (mod 2^63), by squaring.
+__host__ __device__ __forceinline__ void lcg_map(uint64_t n, uint64_t &A, uint64_t &C) {
     uint64_t mul = 2806196910506780709ULL, add = 1ULL;       // current power of the map
     uint64_t acc_mul = 1ULL, acc_add = 0ULL;                  // accumulated map
     n &= 0x7FFFFFFFFFFFFFFFULL;
@@ -31,7 +31,18 @@ __device__ __forceinline__ uint64_t lcg_jump(uint64_t seed, uint64_t n) {
         mul = mul * mul;
         n >>= 1;
     }
-    return (acc_mul * seed + acc_add) & 0x7FFFFFFFFFFFFFFFULL;
+    A = acc_mul;
+    C = acc_add;
+}
+// Jump ahead n steps (arithmetic mod 2^64 then masked: 2^63 divides 2^64, so
+// composing maps this way is exact mod 2^63).
+__device__ __forceinline__ uint64_t lcg_jump(uint64_t seed, uint64_t n) {
+    uint64_t A, C;
+    lcg_map(n, A, C);
+    return (A * seed + C) & 0x7FFFFFFFFFFFFFFFULL;
+}
+__device__ __forceinline__ uint64_t lcg_apply(uint64_t A, uint64_t C, uint64_t s) {
+    return (A * s + C) & 0x7FFFFFFFFFFFFFFFULL;
 }
 // Material draw: cumulative thresholds built in XSBench's order
 // (dist[i] + dist[i-1] + ... + dist[1]); P(material 0) is the remainder.

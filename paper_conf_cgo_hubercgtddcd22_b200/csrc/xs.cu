@@ -397,16 +397,20 @@ __device__ __forceinline__ void store_rec(SortRec *d, const SortRec &r) {
     *reinterpret_cast<uint4 *>(d) =
         make_uint4(r.k, r.mu, (uint32_t)__double2loint(r.E), (uint32_t)__double2hiint(r.E));
 }
+// grid-stride over the lookups; a thread's next lookup is `stride` further,
+// so its state advances by the precomputed map of 2*stride steps (exact)
 __global__ void k_sort_sample(Params P, SortRec *__restrict__ rec, uint32_t *__restrict__ key,
-                              uint32_t *__restrict__ hist) {
+                              uint32_t *__restrict__ hist, uint64_t A2s, uint64_t C2s) {
     using KN = Cfg<NATIVE, PL_STACK, true, 128>;
+    if (P.req) { P.first = P.req->first; P.seed = P.req->seed; }
     const int64_t nu = P.grid_type == 0 ? P.n_union : (P.grid_type == 2 ? P.hash_bins : 1);
-    for (uint64_t k = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; k < P.n;
-         k += (uint64_t)gridDim.x * blockDim.x) {
+    const uint64_t k0 = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    uint64_t st = smp::lcg_jump(P.seed, 2ULL * (P.first + k0));
+    for (uint64_t k = k0; k < P.n; k += (uint64_t)gridDim.x * blockDim.x, st = smp::lcg_apply(A2s, C2s, st)) {
         double E;
         int mat;
         int64_t u;
-        sample<KN>(P, P.first + k, E, mat, u);
+        sample_state<KN>(P, st, E, mat, u);
         // the nuclide grid has no u: bucket by energy (the same monotone role)
         const uint32_t kk = P.grid_type == 1
                                 ? sort_key((uint32_t)mat, (uint32_t)(E * (double)kSortBuckets), (int64_t)kSortBuckets)
@@ -484,31 +488,109 @@ extern "C" uint64_t gtr_xs_sorted_workspace_bytes(uint64_t n) {
     return 36u * n + 4u * (uint64_t)(xs::kSortBins + xs::kScanBlocks);
 }
 
+// the sampling pass and the sort into the workspace (rec0 = the sorted records)
+static int sort_pass(gtr_ctx *ctx, const gtr_launch_cfg *cfg, const xs::Params &P, uint64_t n, void *d_workspace,
+                     uint64_t workspace_bytes, cudaStream_t s) {
+    if (n > 0xFFFFFFFFull || workspace_bytes < gtr_xs_sorted_workspace_bytes(n) ||
+        (reinterpret_cast<uintptr_t>(d_workspace) & 15u) || (uint64_t)P.n_union >= (1ull << 28) ||
+        (cfg && (cfg->flags & GTR_F_HISTORY)))
+        return GTR_EINVAL;
+    if (cfg && !valid_cfg(cfg)) return GTR_EINVAL;
+    xs::SortRec *rec0 = static_cast<xs::SortRec *>(d_workspace), *rec1 = rec0 + n;
+    uint32_t *key = reinterpret_cast<uint32_t *>(rec1 + n), *hist = key + n;
+    GTR_CUDA_TRY(cudaMemsetAsync(hist, 0, 4u * xs::kSortBins, s));
+    const int sb = grid_blocks(ctx, (int64_t)n, 256);
+    uint64_t A2s, C2s;
+    smp::lcg_map(2ULL * (uint64_t)sb * 256u, A2s, C2s);
+    xs::k_sort_sample<<<sb, 256, 0, s>>>(P, rec0, key, hist, A2s, C2s);
+    xs::k_sort_scan_local<<<xs::kScanBlocks, 1024, 0, s>>>(hist, hist + xs::kSortBins);
+    xs::k_sort_scan_add<<<xs::kScanBlocks, 1024, 0, s>>>(hist, hist + xs::kSortBins);
+    xs::k_sort_scatter<<<grid_blocks(ctx, (int64_t)n, 256), 256, 0, s>>>(n, key, rec0, hist, rec1);
+    xs::k_sort_rank<<<grid_blocks(ctx, (int64_t)n, 256), 256, 0, s>>>(n, key, hist, rec1, rec0);
+    GTR_CUDA_TRY(cudaGetLastError());
+    return GTR_OK;
+}
+// the lookups in sorted order from a sorted workspace
+static int presorted_pass(gtr_ctx *ctx, const gtr_launch_cfg *cfg, xs::Params P, uint64_t n, void *d_workspace,
+                          uint64_t workspace_bytes, cudaStream_t s) {
+    if (n > 0xFFFFFFFFull || workspace_bytes < gtr_xs_sorted_workspace_bytes(n) ||
+        (reinterpret_cast<uintptr_t>(d_workspace) & 15u) || (cfg->flags & GTR_F_HISTORY))
+        return GTR_EINVAL;
+    P.s_rec = static_cast<const xs::SortRec *>(d_workspace);
+    xs::LaunchArgs a{ctx, cfg, P, s, nullptr};
+    return xs::launch(a);
+}
+// the sampling pass, the sort and the lookups in sorted order; P carries the
+// outputs (d_out / verify / peer buffers) and, for the host-request form, req
+static int sorted_launch(gtr_ctx *ctx, const gtr_launch_cfg *cfg, xs::Params P, uint64_t n, void *d_workspace,
+                         uint64_t workspace_bytes, cudaStream_t s) {
+    const int st = sort_pass(ctx, cfg, P, n, d_workspace, workspace_bytes, s);
+    if (st) return st;
+    return presorted_pass(ctx, cfg, P, n, d_workspace, workspace_bytes, s);
+}
+
+extern "C" int gtr_xs_sort_lookups(gtr_ctx *ctx, const gtr_xs_tables *tables, uint64_t first, uint64_t n,
+                                   uint64_t seed, void *d_workspace, uint64_t workspace_bytes, void *stream) {
+    if (!ctx || !tables_ok(tables) || !d_workspace) return GTR_EINVAL;
+    if (n == 0) return GTR_OK;
+    return sort_pass(ctx, nullptr, xs::make_params(tables, first, n, seed, nullptr, nullptr, nullptr), n,
+                     d_workspace, workspace_bytes, static_cast<cudaStream_t>(stream));
+}
+
+extern "C" int gtr_xs_lookup_presorted(gtr_ctx *ctx, const gtr_launch_cfg *cfg, const gtr_xs_tables *tables,
+                                       uint64_t first, uint64_t n, uint64_t *d_out, const gtr_xs_verify *verify,
+                                       const void *d_workspace, uint64_t workspace_bytes, void *stream) {
+    if (!ctx || !cfg || !tables_ok(tables) || !d_out || !d_workspace) return GTR_EINVAL;
+    if (n == 0) return GTR_OK;
+    return presorted_pass(ctx, cfg, xs::make_params(tables, first, n, 0, d_out, verify, nullptr), n,
+                          const_cast<void *>(d_workspace), workspace_bytes, static_cast<cudaStream_t>(stream));
+}
+
 extern "C" int gtr_xs_lookup_sorted(gtr_ctx *ctx, const gtr_launch_cfg *cfg, const gtr_xs_tables *tables,
                                     uint64_t first, uint64_t n, uint64_t seed, uint64_t *d_out,
                                     const gtr_xs_verify *verify, void *d_workspace, uint64_t workspace_bytes,
                                     void *stream) {
     if (!ctx || !cfg || !tables_ok(tables) || !d_out || !d_workspace) return GTR_EINVAL;
     if (n == 0) return GTR_OK;
-    if (n > 0xFFFFFFFFull || workspace_bytes < gtr_xs_sorted_workspace_bytes(n) ||
-        (reinterpret_cast<uintptr_t>(d_workspace) & 15u) || (uint64_t)tables->n_union >= (1ull << 28) ||
-        (cfg->flags & GTR_F_HISTORY))
+    return sorted_launch(ctx, cfg, xs::make_params(tables, first, n, seed, d_out, verify, nullptr), n, d_workspace,
+                         workspace_bytes, static_cast<cudaStream_t>(stream));
+}
+
+extern "C" int gtr_xs_lookup_presorted_peers(gtr_ctx *ctx, const gtr_launch_cfg *cfg, const gtr_xs_tables *tables,
+                                             uint64_t first, uint64_t n, uint64_t *const *h_peer_outs, int32_t n_peers,
+                                             const void *d_workspace, uint64_t workspace_bytes, void *stream) {
+    if (!ctx || !cfg || !tables_ok(tables) || !h_peer_outs || n_peers < 1 || n_peers > 8 || !d_workspace)
         return GTR_EINVAL;
-    if (!valid_cfg(cfg)) return GTR_EINVAL;
+    for (int p = 0; p < n_peers; p++)
+        if (!h_peer_outs[p]) return GTR_EINVAL;
+    if (n == 0) return GTR_OK;
+    xs::Params P = xs::make_params(tables, first, n, 0, h_peer_outs[0], nullptr, nullptr);
+    P.n_peers = n_peers;
+    for (int p = 0; p < n_peers; p++) P.peer_out[p] = reinterpret_cast<unsigned long long *>(h_peer_outs[p]);
+    return presorted_pass(ctx, cfg, P, n, const_cast<void *>(d_workspace), workspace_bytes,
+                          static_cast<cudaStream_t>(stream));
+}
+
+extern "C" int gtr_xs_lookup_sorted_host(gtr_ctx *ctx, const gtr_launch_cfg *cfg, const gtr_xs_tables *tables,
+                                         const gtr_xs_request *h_req, uint64_t *h_out, void *d_workspace,
+                                         uint64_t workspace_bytes, void *stream) {
+    if (!ctx || !cfg || !tables_ok(tables) || !h_req || !h_out || !d_workspace) return GTR_EINVAL;
     cudaStream_t s = static_cast<cudaStream_t>(stream);
-    xs::SortRec *rec0 = static_cast<xs::SortRec *>(d_workspace), *rec1 = rec0 + n;
-    uint32_t *key = reinterpret_cast<uint32_t *>(rec1 + n), *hist = key + n;
-    xs::Params P = xs::make_params(tables, first, n, seed, d_out, verify, nullptr);
-    GTR_CUDA_TRY(cudaMemsetAsync(hist, 0, 4u * xs::kSortBins, s));
-    xs::k_sort_sample<<<grid_blocks(ctx, (int64_t)n, 256), 256, 0, s>>>(P, rec0, key, hist);
-    xs::k_sort_scan_local<<<xs::kScanBlocks, 1024, 0, s>>>(hist, hist + xs::kSortBins);
-    xs::k_sort_scan_add<<<xs::kScanBlocks, 1024, 0, s>>>(hist, hist + xs::kSortBins);
-    xs::k_sort_scatter<<<grid_blocks(ctx, (int64_t)n, 256), 256, 0, s>>>(n, key, rec0, hist, rec1);
-    xs::k_sort_rank<<<grid_blocks(ctx, (int64_t)n, 256), 256, 0, s>>>(n, key, hist, rec1, rec0);
-    GTR_CUDA_TRY(cudaGetLastError());
-    P.s_rec = rec0;
-    xs::LaunchArgs a{ctx, cfg, P, s, nullptr};
-    return xs::launch(a);
+    gtr_xs_request *d_req = static_cast<gtr_xs_request *>(ctx->d_stage);
+    uint64_t *d_out = reinterpret_cast<uint64_t *>(static_cast<char *>(ctx->d_stage) + 64);
+    GTR_CUDA_TRY(cudaMemcpyAsync(d_req, h_req, sizeof(gtr_xs_request), cudaMemcpyHostToDevice, s));
+    GTR_CUDA_TRY(cudaMemsetAsync(d_out, 0, 18 * sizeof(uint64_t), s));
+    if (h_req->n) {
+        // the kernels read (first, seed) from d_req; n sizes the launches and the workspace
+        const int st = sorted_launch(ctx, cfg,
+                                     xs::make_params(tables, h_req->first, h_req->n, h_req->seed, d_out, nullptr,
+                                                     d_req),
+                                     h_req->n, d_workspace, workspace_bytes, s);
+        if (st) return st;
+    }
+    GTR_CUDA_TRY(cudaMemcpyAsync(h_out, d_out, 18 * sizeof(uint64_t), cudaMemcpyDeviceToHost, s));
+    GTR_CUDA_TRY(cudaStreamSynchronize(s));
+    return GTR_OK;
 }
 
 extern "C" int gtr_xs_lookup_peers(gtr_ctx *ctx, const gtr_launch_cfg *cfg, const gtr_xs_tables *tables,

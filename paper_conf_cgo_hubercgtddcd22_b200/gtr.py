@@ -111,9 +111,16 @@ _proto = {
     "gtr_xs_sorted_workspace_bytes": (_u64, [_u64]),
     "gtr_xs_lookup_sorted": (_i, [_vp, _P(gtr_launch_cfg), _P(gtr_xs_tables), _u64, _u64, _u64, _vp,
                                   _P(gtr_xs_verify), _vp, _u64, _vp]),
+    "gtr_xs_sort_lookups": (_i, [_vp, _P(gtr_xs_tables), _u64, _u64, _u64, _vp, _u64, _vp]),
+    "gtr_xs_lookup_presorted": (_i, [_vp, _P(gtr_launch_cfg), _P(gtr_xs_tables), _u64, _u64, _vp,
+                                     _P(gtr_xs_verify), _vp, _u64, _vp]),
     "gtr_xs_lookup_peers": (_i, [_vp, _P(gtr_launch_cfg), _P(gtr_xs_tables), _u64, _u64, _u64, _P(_u64), C.c_int32,
                                  _vp]),
     "gtr_xs_lookup_host": (_i, [_vp, _P(gtr_launch_cfg), _P(gtr_xs_tables), _P(gtr_xs_request), _vp, _vp]),
+    "gtr_xs_lookup_presorted_peers": (_i, [_vp, _P(gtr_launch_cfg), _P(gtr_xs_tables), _u64, _u64, _P(_u64),
+                                           C.c_int32, _vp, _u64, _vp]),
+    "gtr_xs_lookup_sorted_host": (_i, [_vp, _P(gtr_launch_cfg), _P(gtr_xs_tables), _P(gtr_xs_request), _vp, _vp,
+                                       _u64, _vp]),
     "gtr_l2_persist": (_i, [_vp, _vp, _u64, _u64, C.c_float, _vp]),
     "gtr_su3_mat_nn": (_i, [_vp, _P(gtr_launch_cfg), _vp, _vp, _vp, _i64, C.c_int32, _vp]),
     "gtr_rs_lookup": (_i, [_vp, _P(gtr_launch_cfg), _P(gtr_rs_tables), _u64, _u64, _u64, _vp,
@@ -286,6 +293,36 @@ def gtr_xs_lookup_peers(ctx, launch_cfg, tables, first, n, seed, peer_ptrs, stre
 def gtr_xs_lookup_host(ctx, launch_cfg, tables, h_req, h_out, stream=None):
     return _check("gtr_xs_lookup_host", _lib.gtr_xs_lookup_host(ctx, C.byref(launch_cfg), C.byref(tables),
                                                                 C.byref(h_req), _ptr(h_out), _stream(stream)))
+
+
+def gtr_xs_sort_lookups(ctx, tables, first, n, seed, d_workspace, stream=None):
+    nbytes = d_workspace.numel() * d_workspace.element_size()
+    return _check("gtr_xs_sort_lookups",
+                  _lib.gtr_xs_sort_lookups(ctx, C.byref(tables), first, n, seed, _ptr(d_workspace), nbytes,
+                                           _stream(stream)))
+
+
+def gtr_xs_lookup_presorted(ctx, launch_cfg, tables, first, n, d_out, d_workspace, verify=None, stream=None):
+    nbytes = d_workspace.numel() * d_workspace.element_size()
+    return _check("gtr_xs_lookup_presorted",
+                  _lib.gtr_xs_lookup_presorted(ctx, C.byref(launch_cfg), C.byref(tables), first, n, _ptr(d_out),
+                                               C.byref(verify) if verify else None, _ptr(d_workspace), nbytes,
+                                               _stream(stream)))
+
+
+def gtr_xs_lookup_presorted_peers(ctx, launch_cfg, tables, first, n, peer_ptrs, d_workspace, stream=None):
+    arr = (_u64 * len(peer_ptrs))(*peer_ptrs)
+    nbytes = d_workspace.numel() * d_workspace.element_size()
+    return _check("gtr_xs_lookup_presorted_peers",
+                  _lib.gtr_xs_lookup_presorted_peers(ctx, C.byref(launch_cfg), C.byref(tables), first, n, arr,
+                                                     len(peer_ptrs), _ptr(d_workspace), nbytes, _stream(stream)))
+
+
+def gtr_xs_lookup_sorted_host(ctx, launch_cfg, tables, h_req, h_out, d_workspace, stream=None):
+    nbytes = d_workspace.numel() * d_workspace.element_size()
+    return _check("gtr_xs_lookup_sorted_host",
+                  _lib.gtr_xs_lookup_sorted_host(ctx, C.byref(launch_cfg), C.byref(tables), C.byref(h_req),
+                                                 _ptr(h_out), _ptr(d_workspace), nbytes, _stream(stream)))
 
 
 def gtr_su3_mat_nn(ctx, launch_cfg, d_A, d_B, d_C, sites, iters, stream=None):

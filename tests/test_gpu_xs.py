@@ -424,6 +424,45 @@ def test_sorted_coherent_dense(G, ctx, dense, cfg, first, n):
     _assert_same(out, v, o_out, o_v)
 
 
+@pytest.mark.parametrize("mode", (0, 2, 3, 4))
+def test_sorted_host_and_peers(G, ctx, dev_small, small, mode):
+    """The sorted event mode through its host-buffer entry point (request
+    copied to the device, results copied back) and with the fused peer
+    combine (the same buffer listed 3 times gets 3 x the oracle)."""
+    t, P, o_out, o_v, n = small
+    c = G.cfg(mode, G.PL_STACK, 1, 256)
+    ws = torch.empty(G.gtr_xs_sorted_workspace_bytes(n), dtype=torch.uint8, device="cuda")
+    h_out = torch.zeros(18, dtype=torch.uint64).pin_memory()
+    G.gtr_xs_lookup_sorted_host(ctx, c, dev_small.tables, G.gtr_xs_request(0, n, X.SEED_L), h_out, ws)
+    G.gtr_ctx_check(ctx)
+    assert np.array_equal(h_out.numpy(), o_out)
+    o2, _ = P.run(777, 5000, X.SEED_L + 9, 4)
+    G.gtr_xs_lookup_sorted_host(ctx, c, dev_small.tables, G.gtr_xs_request(777, 5000, X.SEED_L + 9), h_out, ws)
+    G.gtr_ctx_check(ctx)
+    assert np.array_equal(h_out.numpy(), o2)
+    buf = torch.zeros(18, dtype=torch.uint64, device="cuda")
+    G.gtr_xs_sort_lookups(ctx, dev_small.tables, 0, n, X.SEED_L, ws)
+    G.gtr_xs_lookup_presorted_peers(ctx, c, dev_small.tables, 0, n, [buf.data_ptr()] * 3, ws)
+    G.gtr_ctx_check(ctx)
+    assert np.array_equal(buf.cpu().numpy(), (o_out * np.uint64(3)).astype(np.uint64))
+
+
+def test_sort_then_presorted(G, ctx, dev_small, small):
+    """The two halves of the sorted mode: one sort, then the presorted
+    lookups in several modes from the same workspace -- each identical to the
+    oracle, per lookup."""
+    t, P, o_out, o_v, n = small
+    ws = torch.empty(G.gtr_xs_sorted_workspace_bytes(n), dtype=torch.uint8, device="cuda")
+    G.gtr_xs_sort_lookups(ctx, dev_small.tables, 0, n, X.SEED_L, ws)
+    for c in (G.cfg(G.SPMD, G.PL_STACK, 1, 256), G.cfg(G.CSM, G.PL_RUNTIME, 0, 128),
+              G.cfg(G.GENERIC, G.PL_STACK, 1, 256), G.cfg(G.NATIVE, G.PL_STACK, 1, 256)):
+        out = torch.zeros(18, dtype=torch.uint64, device="cuda")
+        v, bufs = dev_small.verify_buffers(n)
+        G.gtr_xs_lookup_presorted(ctx, c, dev_small.tables, 0, n, out, ws, v)
+        G.gtr_ctx_check(ctx)
+        _assert_same(out.cpu().numpy(), {k: b.cpu().numpy() for k, b in bufs.items()}, o_out, o_v)
+
+
 def test_sorted_mode_rejects_small_workspace(G, ctx, dev_small):
     out = torch.zeros(18, dtype=torch.uint64, device="cuda")
     ws = torch.empty(1024, dtype=torch.uint8, device="cuda")
