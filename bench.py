@@ -614,7 +614,11 @@ def sweeps(G, torch, ctx, xs, first, seed, stream, cpu=True):
                              ("spmd_sorted", G.cfg(G.SPMD, G.PL_STACK, 1, 256), True),
                              ("csm_sorted", G.cfg(G.CSM, G.PL_STACK, 1, 256), True),
                              ("generic_sorted", G.cfg(G.GENERIC, G.PL_STACK, 1, 256), True),
-                             ("native_sorted", G.cfg(G.NATIVE, G.PL_STACK, 1, 256), True)]:
+                             ("native_sorted", G.cfg(G.NATIVE, G.PL_STACK, 1, 256), True),
+                             # the CUDA watermark of the sorted schedule: the same warp-coherent
+                             # loops as a plain CUDA kernel (no runtime)
+                             ("native_coherent_sorted",
+                              G.cfg(G.NATIVE, G.PL_STACK, 1, 256, flags=G.F_NATIVE_BUCKETED), True)]:
         def f():
             out.zero_()
             if sorted_:
@@ -625,6 +629,8 @@ def sweeps(G, torch, ctx, xs, first, seed, stream, cpu=True):
         f2[name] = {"lookups_per_s": n / (ms * 1e-3), "ms": ms,
                     "same_result": bool(np.array_equal(out.cpu().numpy(), ref))}
     del ws
+    f2["fraction_of_cuda_sorted"] = {m: f2[m + "_sorted"]["lookups_per_s"] / f2["native_coherent_sorted"]["lookups_per_s"]
+                                     for m in ("spmd", "csm", "generic")}
     # the paper's ladder (Fig. 11a) on SPMD: globalized at runtime -> h2s2 -> +fold
     ladder = {}
     for name, c in [("llvm12_coalesced", G.cfg(G.SPMD, G.PL_COALESCED, 0, 256)),

@@ -17,6 +17,7 @@ import sys
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 sys.path.insert(0, ROOT)
 
+import numpy as np
 import torch  # noqa: E402
 
 import gtr_inputs.rs as RS  # noqa: E402
@@ -82,10 +83,32 @@ if parts & {"xs", "xs_grids", "xs_sorted", "xs_peers"}:
         ran.append("xs_grids")
     if "xs_sorted" in parts:
         ws = torch.empty(G.gtr_xs_sorted_workspace_bytes(3000), dtype=torch.uint8, device="cuda")
-        for m, p, f, fl in ((G.SPMD, G.PL_STACK, 1, 0), (G.CSM, G.PL_RUNTIME, 0, 0), (G.GENERIC, G.PL_STACK, 1, 0),
-                            (G.SPMD, G.PL_STACK, 1, G.F_PLAIN), (G.NATIVE, G.PL_STACK, 1, 0)):
-            G.gtr_xs_lookup_sorted(ctx, G.cfg(m, p, f, 128, num_teams=teams, flags=fl), xs.tables, 0, 3000, X.SEED_L,
+        for m, p, f, fl, nt in ((G.SPMD, G.PL_STACK, 1, 0, 128), (G.CSM, G.PL_RUNTIME, 0, 0, 128),
+                                (G.GENERIC, G.PL_STACK, 1, 0, 128), (G.SPMD, G.PL_STACK, 1, G.F_PLAIN, 128),
+                                (G.NATIVE, G.PL_STACK, 1, 0, 128), (G.SPMD, G.PL_STACK, 1, 0, 256),
+                                (G.CSM, G.PL_STACK, 1, 0, 256), (G.NATIVE, G.PL_STACK, 1, G.F_NATIVE_BUCKETED, 256)):
+            G.gtr_xs_lookup_sorted(ctx, G.cfg(m, p, f, nt, num_teams=teams, flags=fl), xs.tables, 0, 3000, X.SEED_L,
                                    u64(18), ws)
+        # the split form and the host-request form (warp-coherent path on a
+        # denser table: 68 nuclides x 200 gridpoints, 20,000 lookups)
+        td = X.make_tables(68, 200)
+        xd = XsDevice(ctx, td)
+        wd = torch.empty(G.gtr_xs_sorted_workspace_bytes(20000), dtype=torch.uint8, device="cuda")
+        G.gtr_xs_sort_lookups(ctx, xd.tables, 5, 20000, X.SEED_L, wd)
+        G.gtr_xs_lookup_presorted(ctx, G.cfg(G.SPMD, G.PL_STACK, 1, 256, num_teams=teams), xd.tables, 5, 20000,
+                                  u64(18), wd)
+        G.gtr_xs_lookup_presorted_peers(ctx, G.cfg(G.CSM, G.PL_STACK, 1, 128, num_teams=teams), xd.tables, 5, 20000,
+                                        [u64(18).data_ptr()], wd)
+        h = torch.zeros(18, dtype=torch.uint64).pin_memory()
+        G.gtr_xs_lookup_sorted_host(ctx, G.cfg(G.SPMD, G.PL_STACK, 1, 256, num_teams=teams), xd.tables,
+                                    G.gtr_xs_request(0, 20000, X.SEED_L), h, wd)
+        # duplicate gridpoint energies: union scatter + sequential-rule index builder
+        tdup = X.make_tables(3, 50)
+        tdup["grid"][0, 11, 0] = tdup["grid"][0, 10, 0]
+        tdup["grid"][1, 30, 0] = tdup["grid"][0, 30, 0]
+        for n_ in range(3):
+            tdup["grid"][n_] = tdup["grid"][n_][np.argsort(tdup["grid"][n_, :, 0], kind="stable")]
+        XsDevice(ctx, tdup)
         ran.append("xs_sorted")
     if "xs_peers" in parts:
         bufs = [u64(18) for _ in range(3)]
