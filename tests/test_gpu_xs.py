@@ -463,6 +463,31 @@ def test_sort_then_presorted(G, ctx, dev_small, small):
         _assert_same(out.cpu().numpy(), {k: b.cpu().numpy() for k, b in bufs.items()}, o_out, o_v)
 
 
+def test_sorted_entry_points_reject_bad_workspace(G, ctx, dev_small):
+    """Synchronous GTR_EINVAL (no launch) for a workspace that is too small or
+    not 16-byte aligned, on every sorted-mode entry point."""
+    n = 1000
+    need = G.gtr_xs_sorted_workspace_bytes(n)
+    small_ws = torch.empty(need - 16, dtype=torch.uint8, device="cuda")
+    big = torch.empty(need + 64, dtype=torch.uint8, device="cuda")
+    misaligned = big[8:8 + need]
+    out = torch.zeros(18, dtype=torch.uint64, device="cuda")
+    h_out = torch.zeros(18, dtype=torch.uint64).pin_memory()
+    c = G.cfg(G.SPMD, G.PL_STACK, 1, 256)
+    for ws in (small_ws, misaligned):
+        calls = [lambda: G.gtr_xs_sort_lookups(ctx, dev_small.tables, 0, n, X.SEED_L, ws),
+                 lambda: G.gtr_xs_lookup_presorted(ctx, c, dev_small.tables, 0, n, out, ws),
+                 lambda: G.gtr_xs_lookup_presorted_peers(ctx, c, dev_small.tables, 0, n, [out.data_ptr()], ws),
+                 lambda: G.gtr_xs_lookup_sorted_host(ctx, c, dev_small.tables, G.gtr_xs_request(0, n, X.SEED_L),
+                                                     h_out, ws),
+                 lambda: G.gtr_xs_lookup_sorted(ctx, c, dev_small.tables, 0, n, X.SEED_L, out, ws)]
+        for call in calls:
+            with pytest.raises(G.GtrError):
+                call()
+    G.gtr_ctx_check(ctx)
+    assert int(out.sum()) == 0
+
+
 def test_sorted_mode_rejects_small_workspace(G, ctx, dev_small):
     out = torch.zeros(18, dtype=torch.uint64, device="cuda")
     ws = torch.empty(1024, dtype=torch.uint8, device="cuda")
