@@ -383,7 +383,10 @@ extern "C" int gtr_xs_lookup_host(gtr_ctx *ctx, const gtr_launch_cfg *cfg, const
 // rec0 holds the samples in lookup order, then the final (ranked) order.
 namespace gtr {
 namespace xs {
-constexpr uint32_t kSortBuckets = 1u << 17;           // u buckets per material
+#ifndef GTR_XS_SORT_LOG2
+#define GTR_XS_SORT_LOG2 17
+#endif
+constexpr uint32_t kSortBuckets = 1u << GTR_XS_SORT_LOG2;   // u buckets per material
 constexpr uint32_t kSortBins = 12u * kSortBuckets;
 constexpr uint32_t kScanBlocks = kSortBins / 1024;
 constexpr uint32_t kRankMax = 256;                    // larger buckets keep the scatter's order
