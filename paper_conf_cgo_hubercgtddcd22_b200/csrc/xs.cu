@@ -144,6 +144,62 @@ __global__ void k_index_sequential(int32_t *__restrict__ idx, int64_t n_union, i
     }
 }
 
+// Self-test of the branch-free interpolation-factor division (ddiv_fast,
+// DESIGN.md R-XS-div): operand pairs from a counter-based hash -- raw 64-bit
+// patterns (every exponent, subnormals, Inf, NaN), pairs of unit-interval
+// energies as the lookups form them, and near-equal / near-overflow pairs --
+// each compared bit for bit with the IEEE division wherever ddiv_fast's
+// guard accepts.  counts[0] += mismatches, counts[1] += accepted pairs.
+__device__ __forceinline__ uint64_t mix64(uint64_t z) {
+    z += 0x9E3779B97F4A7C15ull;
+    z = (z ^ (z >> 30)) * 0xBF58476D1CE4E5B9ull;
+    z = (z ^ (z >> 27)) * 0x94D049BB133111EBull;
+    return z ^ (z >> 31);
+}
+__global__ void k_ddiv_selftest(uint64_t n, uint64_t seed, unsigned long long *counts) {
+    unsigned long long bad = 0, acc = 0;
+    for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (uint64_t)gridDim.x * blockDim.x) {
+        const uint64_t a = mix64(seed ^ (2 * i)), b = mix64(seed ^ (2 * i + 1));
+        double x, y;
+        switch (i & 3) {
+        case 0:                                        // raw bit patterns
+            x = __longlong_as_double((long long)a);
+            y = __longlong_as_double((long long)b);
+            break;
+        case 1: {                                      // (hi.e - E) / (hi.e - lo.e), energies in [0, 1)
+            const double e0 = (double)(a >> 11) * 0x1p-53, e1 = (double)(b >> 11) * 0x1p-53;
+            const double lo = fmin(e0, e1), hi = fmax(e0, e1);
+            const double E = lo + (hi - lo) * ((double)(mix64(a ^ b) >> 11) * 0x1p-53);
+            x = hi - E;
+            y = hi - lo;
+            break;
+        }
+        case 2: {                                      // neighbouring doubles: tiny denominators
+            const double e = (double)(a >> 11) * 0x1p-53;
+            const double h = __longlong_as_double(__double_as_longlong(e) + (long long)(1 + (b & 7)));
+            x = h - (double)((b >> 8) >> 11) * 0x1p-53 * (h - e);
+            y = h - e;
+            break;
+        }
+        default: {                                     // random exponents across the whole range
+            x = ldexp(1.0 + (double)(a >> 12) * 0x1p-52, (int)(a & 2047) - 1075);
+            y = ldexp(1.0 + (double)(b >> 12) * 0x1p-52, (int)(b & 2047) - 1075);
+            if (b & 0x800) y = -y;
+        }
+        }
+        bool ok;
+        const double q = xs::ddiv_fast(x, y, ok);
+        if (ok) {
+            acc++;
+            const double r = x / y;
+            const bool same = (__double_as_longlong(q) == __double_as_longlong(r)) || (q != q && r != r);
+            if (!same) bad++;
+        }
+    }
+    if (bad) atomicAdd(counts, bad);
+    atomicAdd(counts + 1, acc);
+}
+
 // Runtime-mode variants: defined (explicitly instantiated) in xs_variant.cu.
 template <class K> int run_variant(LaunchArgs &a);
 template <class K> struct VariantOp {
@@ -215,6 +271,15 @@ int gtr_internal_query_xs(gtr_ctx *ctx, const gtr_launch_cfg *cfg, gtr_variant_i
     gtr_xs_tables t = {};
     xs::LaunchArgs a{ctx, cfg, xs::make_params(&t, 0, 0, 0, nullptr, nullptr, nullptr), nullptr, info};
     return xs::launch(a);
+}
+
+extern "C" int gtr_ddiv_selftest(gtr_ctx *ctx, uint64_t n, uint64_t seed, uint64_t *d_counts, void *stream) {
+    if (!ctx || !d_counts) return GTR_EINVAL;
+    if (n == 0) return GTR_OK;
+    xs::k_ddiv_selftest<<<ctx->num_sms * 8, 256, 0, static_cast<cudaStream_t>(stream)>>>(
+        n, seed, reinterpret_cast<unsigned long long *>(d_counts));
+    GTR_CUDA_TRY(cudaGetLastError());
+    return GTR_OK;
 }
 
 extern "C" uint64_t gtr_xs_build_workspace_bytes(int64_t n_iso, int64_t n_gp) {

@@ -98,6 +98,7 @@ _proto = {
     "gtr_forkjoin": (_i, [_vp, _P(gtr_launch_cfg), _i64, C.c_int32, C.c_int32, _vp, _vp]),
     "gtr_barrier_floor": (_i, [_vp, _P(gtr_launch_cfg), _i64, _vp, _vp]),
     "gtr_fp64_probe": (_i, [_vp, _i64, _vp, _P(C.c_double), _vp]),
+    "gtr_ddiv_selftest": (_i, [_vp, _u64, _u64, _vp, _vp]),
     "gtr_semantics": (_i, [_vp, _P(gtr_launch_cfg), C.c_int32, _vp, _i64, _vp]),
     "gtr_xs_build_workspace_bytes": (_u64, [_i64, _i64]),
     "gtr_xs_build_egrid": (_i, [_vp, _vp, _i64, _i64, _vp, _vp, _vp]),
@@ -213,6 +214,10 @@ def gtr_forkjoin(ctx, launch_cfg, regions, body, n_distinct, d_out, stream=None)
 def gtr_barrier_floor(ctx, launch_cfg, iters, d_out, stream=None):
     return _check("gtr_barrier_floor", _lib.gtr_barrier_floor(ctx, C.byref(launch_cfg), iters, _ptr(d_out),
                                                               _stream(stream)))
+
+
+def gtr_ddiv_selftest(ctx, n, seed, d_counts, stream=None):
+    return _check("gtr_ddiv_selftest", _lib.gtr_ddiv_selftest(ctx, n, seed, _ptr(d_counts), _stream(stream)))
 
 
 def gtr_fp64_probe(ctx, iters, d_out, stream=None):

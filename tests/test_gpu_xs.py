@@ -447,6 +447,20 @@ def test_sorted_host_and_peers(G, ctx, dev_small, small, mode):
     assert np.array_equal(buf.cpu().numpy(), (o_out * np.uint64(3)).astype(np.uint64))
 
 
+def test_branch_free_division_matches_ieee(G, ctx):
+    """R-XS-div: wherever its guard accepts, the branch-free division of the
+    warp-coherent loops returns exactly the IEEE quotient -- 2^28 pairs of raw
+    bit patterns, lookup-shaped energy differences, neighbouring doubles and
+    random exponents; the guard accepts the lookup-shaped pairs."""
+    counts = torch.zeros(2, dtype=torch.uint64, device="cuda")
+    n = 1 << 28
+    G.gtr_ddiv_selftest(ctx, n, 20221002, counts)
+    G.gtr_ctx_check(ctx)
+    bad, acc = (int(x) for x in counts.cpu())
+    assert bad == 0
+    assert acc > n // 2          # all of the energy-shaped quarter and most of the rest
+
+
 def test_sort_then_presorted(G, ctx, dev_small, small):
     """The two halves of the sorted mode: one sort, then the presorted
     lookups in several modes from the same workspace -- each identical to the
