@@ -39,7 +39,7 @@ FLOPS_PER_NUCLIDE = 28      # fp64 ops of one nuclide visit (c3.2), a division c
 def parse():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
-    ap.add_argument("--steps", type=int, default=20)
+    ap.add_argument("--steps", type=int, default=100)   # ~0.5 s timed: several clock samples
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="gtr", choices=["gtr", "reference"])
     ap.add_argument("--no-sweep", action="store_true", help="skip the per-mode / fork-join sweeps")
