@@ -440,14 +440,18 @@ extern "C" int gtr_xs_lookup_host(gtr_ctx *ctx, const gtr_launch_cfg *cfg, const
 // rows), which the warp-coherent nuclide loops (CoherentRegion) exploit.
 // Results are identical: each lookup's arithmetic is its own, the tallies
 // are sums.  The sort: counting sort by (material, u bucket) with 2^17
-// buckets per material, then each bucket (fuel: ~18 lookups) ordered by
-// (u, lookup) with a rank count -- a warp's 32 lookups then span ~50 union
-// points instead of a whole bucket.  Workspace (caller-owned,
+// buckets per material (fuel: ~18 lookups, ~30 union points per bucket), so
+// a warp's 32 lookups span ~2-3 buckets.  GTR_XS_SORT_RANK=1 additionally
+// orders each bucket by (u, lookup) with a rank count (a deterministic order;
+// measured: the lookups gain 2%, the rank pass costs 6% of the step).  Workspace (caller-owned,
 // gtr_xs_sorted_workspace_bytes), 16-byte aligned:
 //   rec0[n] SortRec | rec1[n] SortRec | key[n] u32 | hist[12*NB] u32 | totals u32
 // rec0 holds the samples in lookup order, then the final (ranked) order.
 namespace gtr {
 namespace xs {
+#ifndef GTR_XS_SORT_RANK
+#define GTR_XS_SORT_RANK 0
+#endif
 #ifndef GTR_XS_SORT_LOG2
 #define GTR_XS_SORT_LOG2 17
 #endif
@@ -570,11 +574,18 @@ static int sort_pass(gtr_ctx *ctx, const gtr_launch_cfg *cfg, const xs::Params &
     const int sb = grid_blocks(ctx, (int64_t)n, 256);
     uint64_t A2s, C2s;
     smp::lcg_map(2ULL * (uint64_t)sb * 256u, A2s, C2s);
+#if GTR_XS_SORT_RANK
     xs::k_sort_sample<<<sb, 256, 0, s>>>(P, rec0, key, hist, A2s, C2s);
     xs::k_sort_scan_local<<<xs::kScanBlocks, 1024, 0, s>>>(hist, hist + xs::kSortBins);
     xs::k_sort_scan_add<<<xs::kScanBlocks, 1024, 0, s>>>(hist, hist + xs::kSortBins);
     xs::k_sort_scatter<<<grid_blocks(ctx, (int64_t)n, 256), 256, 0, s>>>(n, key, rec0, hist, rec1);
     xs::k_sort_rank<<<grid_blocks(ctx, (int64_t)n, 256), 256, 0, s>>>(n, key, hist, rec1, rec0);
+#else   // bucket order only (no in-bucket ranking): samples in rec1, the scatter into rec0
+    xs::k_sort_sample<<<sb, 256, 0, s>>>(P, rec1, key, hist, A2s, C2s);
+    xs::k_sort_scan_local<<<xs::kScanBlocks, 1024, 0, s>>>(hist, hist + xs::kSortBins);
+    xs::k_sort_scan_add<<<xs::kScanBlocks, 1024, 0, s>>>(hist, hist + xs::kSortBins);
+    xs::k_sort_scatter<<<grid_blocks(ctx, (int64_t)n, 256), 256, 0, s>>>(n, key, rec1, hist, rec0);
+#endif
     GTR_CUDA_TRY(cudaGetLastError());
     return GTR_OK;
 }
