@@ -524,8 +524,9 @@ def run_gtr(a):
                     "note": ("gtr_xs_lookup_sorted_host" if sorted_ else "gtr_xs_lookup_host") +
                             ": pinned host request -> device, lookups, 18 u64 -> pinned host, "
                             "stream sync; tables resident (uploaded once, table_setup_s)"},
-            # our kernels per step: sampling, 2 scan, scatter, rank, lookups (sorted); the lookups (bucketed)
-            "gpu_launches": a.steps * (6 if sorted_ else 1),
+            # our kernels per step: sampling, 2 scan, scatter, lookups (sorted; a GTR_XS_SORT_RANK=1 build
+            # adds the rank pass); the lookups (bucketed)
+            "gpu_launches": a.steps * (5 if sorted_ else 1),
             "clocks": clk.summary(),
             "host": host_info(),
         }
