@@ -226,6 +226,17 @@ def xs_small_config(G, torch, ctx, stream):
         ms = _time(torch, stream, f, 5)
         res[name] = {"lookups_per_s": n / (ms * 1e-3), "ms": ms,
                      "same_result_as_oracle": bool(np.array_equal(out.cpu().numpy(), o1))}
+    # the sorted event mode at this size (sort + presorted lookups in one call)
+    ws = torch.empty(G.gtr_xs_sorted_workspace_bytes(n), dtype=torch.uint8, device="cuda")
+    c = G.cfg(G.SPMD, G.PL_STACK, 1, 256)
+
+    def fs():
+        out.zero_()
+        G.gtr_xs_lookup_sorted(ctx, c, xs.tables, 0, n, X.SEED_L, out, ws, None, stream)
+    ms = _time(torch, stream, fs, 5)
+    res["spmd_sorted"] = {"lookups_per_s": n / (ms * 1e-3), "ms": ms,
+                          "same_result_as_oracle": bool(np.array_equal(out.cpu().numpy(), o1))}
+    del ws
     res["cpu_oracle_1core"] = {"lookups_per_s": n / d1, "cores": 1, "kind": "oracle", "sample": "full run"}
     res["cpu_oracle_nproc"] = {"lookups_per_s": n / dn, "cores": cores, "kind": "oracle", "sample": "full run"}
     del xs
@@ -614,6 +625,7 @@ def sweeps(G, torch, ctx, xs, first, seed, stream, cpu=True):
                              ("native_history", G.cfg(G.NATIVE, G.PL_STACK, 1, 256, flags=G.F_HISTORY), False),
                              ("spmd_sorted", G.cfg(G.SPMD, G.PL_STACK, 1, 256), True),
                              ("csm_sorted", G.cfg(G.CSM, G.PL_STACK, 1, 256), True),
+                             ("cascade_sorted", G.cfg(G.GENERIC_CASCADE, G.PL_STACK, 1, 256), True),
                              ("generic_sorted", G.cfg(G.GENERIC, G.PL_STACK, 1, 256), True),
                              ("native_sorted", G.cfg(G.NATIVE, G.PL_STACK, 1, 256), True),
                              # the CUDA watermark of the sorted schedule: the same warp-coherent
@@ -631,7 +643,7 @@ def sweeps(G, torch, ctx, xs, first, seed, stream, cpu=True):
                     "same_result": bool(np.array_equal(out.cpu().numpy(), ref))}
     del ws
     f2["fraction_of_cuda_sorted"] = {m: f2[m + "_sorted"]["lookups_per_s"] / f2["native_coherent_sorted"]["lookups_per_s"]
-                                     for m in ("spmd", "csm", "generic")}
+                                     for m in ("spmd", "csm", "cascade", "generic")}
     # the paper's ladder (Fig. 11a) on SPMD: globalized at runtime -> h2s2 -> +fold
     ladder = {}
     for name, c in [("llvm12_coalesced", G.cfg(G.SPMD, G.PL_COALESCED, 0, 256)),
