@@ -455,15 +455,22 @@ namespace xs {
 #ifndef GTR_XS_SORT_LOG2
 #define GTR_XS_SORT_LOG2 17
 #endif
-constexpr uint32_t kSortBuckets = 1u << GTR_XS_SORT_LOG2;   // u buckets per material
-constexpr uint32_t kSortBins = 12u * kSortBuckets;
-constexpr uint32_t kScanBlocks = kSortBins / 1024;
+// u buckets per material: 2^lg with lg = ceil(log2(n / 128)) clamped to
+// [8, GTR_XS_SORT_LOG2] -- ~128 lookups per bucket row of 12 materials, so a
+// small request does not pay for a 1.57M-bin histogram (17M lookups: 2^17)
+inline uint32_t sort_log2(uint64_t n) {
+    uint32_t lg = 8;
+    while (lg < GTR_XS_SORT_LOG2 && (128ull << lg) < n) lg++;
+    return lg;
+}
+inline uint64_t sort_bins(uint64_t n) { return 12ull << sort_log2(n); }   // a multiple of 1024 (lg >= 8)
 constexpr uint32_t kRankMax = 256;                    // larger buckets keep the scatter's order
 
-__device__ __forceinline__ uint32_t sort_key(uint32_t mat, uint32_t u, int64_t n_union) {
-    uint32_t b = (uint32_t)(((uint64_t)u * kSortBuckets) / (uint64_t)n_union);
-    b = b < kSortBuckets ? b : kSortBuckets - 1;
-    return mat * kSortBuckets + b;
+__device__ __forceinline__ uint32_t sort_key(uint32_t mat, uint32_t u, int64_t n_union, uint32_t lg) {
+    const uint32_t nb = 1u << lg;
+    uint32_t b = (uint32_t)(((uint64_t)u << lg) / (uint64_t)n_union);
+    b = b < nb ? b : nb - 1;
+    return mat * nb + b;
 }
 __device__ __forceinline__ void store_rec(SortRec *d, const SortRec &r) {
     *reinterpret_cast<uint4 *>(d) =
@@ -472,7 +479,7 @@ __device__ __forceinline__ void store_rec(SortRec *d, const SortRec &r) {
 // grid-stride over the lookups; a thread's next lookup is `stride` further,
 // so its state advances by the precomputed map of 2*stride steps (exact)
 __global__ void k_sort_sample(Params P, SortRec *__restrict__ rec, uint32_t *__restrict__ key,
-                              uint32_t *__restrict__ hist, uint64_t A2s, uint64_t C2s) {
+                              uint32_t *__restrict__ hist, uint64_t A2s, uint64_t C2s, uint32_t lg) {
     using KN = Cfg<NATIVE, PL_STACK, true, 128>;
     if (P.req) { P.first = P.req->first; P.seed = P.req->seed; }
     const int64_t nu = P.grid_type == 0 ? P.n_union : (P.grid_type == 2 ? P.hash_bins : 1);
@@ -485,8 +492,8 @@ __global__ void k_sort_sample(Params P, SortRec *__restrict__ rec, uint32_t *__r
         sample_state<KN>(P, st, E, mat, u);
         // the nuclide grid has no u: bucket by energy (the same monotone role)
         const uint32_t kk = P.grid_type == 1
-                                ? sort_key((uint32_t)mat, (uint32_t)(E * (double)kSortBuckets), (int64_t)kSortBuckets)
-                                : sort_key((uint32_t)mat, (uint32_t)u, nu);
+                                ? sort_key((uint32_t)mat, (uint32_t)(E * (double)(1u << lg)), (int64_t)(1u << lg), lg)
+                                : sort_key((uint32_t)mat, (uint32_t)u, nu, lg);
         key[k] = kk;
         SortRec r;
         r.k = (uint32_t)k;
@@ -496,7 +503,7 @@ __global__ void k_sort_sample(Params P, SortRec *__restrict__ rec, uint32_t *__r
         atomicAdd(hist + kk, 1u);
     }
 }
-// exclusive scan of hist[kSortBins] in place: per 1024-bin block a shared-
+// exclusive scan of hist[bins] in place: per 1024-bin block a shared-
 // memory scan + the block total, then every block adds the totals before it
 __global__ void __launch_bounds__(1024) k_sort_scan_local(uint32_t *hist, uint32_t *totals) {
     __shared__ uint32_t part[1024];
@@ -557,7 +564,7 @@ __global__ void k_sort_rank(uint64_t n, const uint32_t *__restrict__ key, const 
 }  // namespace gtr
 
 extern "C" uint64_t gtr_xs_sorted_workspace_bytes(uint64_t n) {
-    return 36u * n + 4u * (uint64_t)(xs::kSortBins + xs::kScanBlocks);
+    return 36u * n + 4u * (xs::sort_bins(n) + xs::sort_bins(n) / 1024u);
 }
 
 // the sampling pass and the sort into the workspace (rec0 = the sorted records)
@@ -570,20 +577,22 @@ static int sort_pass(gtr_ctx *ctx, const gtr_launch_cfg *cfg, const xs::Params &
     if (cfg && !valid_cfg(cfg)) return GTR_EINVAL;
     xs::SortRec *rec0 = static_cast<xs::SortRec *>(d_workspace), *rec1 = rec0 + n;
     uint32_t *key = reinterpret_cast<uint32_t *>(rec1 + n), *hist = key + n;
-    GTR_CUDA_TRY(cudaMemsetAsync(hist, 0, 4u * xs::kSortBins, s));
+    const uint32_t lg = xs::sort_log2(n);
+    const uint32_t bins = (uint32_t)xs::sort_bins(n), blocks = bins / 1024u;
+    GTR_CUDA_TRY(cudaMemsetAsync(hist, 0, 4u * bins, s));
     const int sb = grid_blocks(ctx, (int64_t)n, 256);
     uint64_t A2s, C2s;
     smp::lcg_map(2ULL * (uint64_t)sb * 256u, A2s, C2s);
 #if GTR_XS_SORT_RANK
-    xs::k_sort_sample<<<sb, 256, 0, s>>>(P, rec0, key, hist, A2s, C2s);
-    xs::k_sort_scan_local<<<xs::kScanBlocks, 1024, 0, s>>>(hist, hist + xs::kSortBins);
-    xs::k_sort_scan_add<<<xs::kScanBlocks, 1024, 0, s>>>(hist, hist + xs::kSortBins);
+    xs::k_sort_sample<<<sb, 256, 0, s>>>(P, rec0, key, hist, A2s, C2s, lg);
+    xs::k_sort_scan_local<<<blocks, 1024, 0, s>>>(hist, hist + bins);
+    xs::k_sort_scan_add<<<blocks, 1024, 0, s>>>(hist, hist + bins);
     xs::k_sort_scatter<<<grid_blocks(ctx, (int64_t)n, 256), 256, 0, s>>>(n, key, rec0, hist, rec1);
     xs::k_sort_rank<<<grid_blocks(ctx, (int64_t)n, 256), 256, 0, s>>>(n, key, hist, rec1, rec0);
 #else   // bucket order only (no in-bucket ranking): samples in rec1, the scatter into rec0
-    xs::k_sort_sample<<<sb, 256, 0, s>>>(P, rec1, key, hist, A2s, C2s);
-    xs::k_sort_scan_local<<<xs::kScanBlocks, 1024, 0, s>>>(hist, hist + xs::kSortBins);
-    xs::k_sort_scan_add<<<xs::kScanBlocks, 1024, 0, s>>>(hist, hist + xs::kSortBins);
+    xs::k_sort_sample<<<sb, 256, 0, s>>>(P, rec1, key, hist, A2s, C2s, lg);
+    xs::k_sort_scan_local<<<blocks, 1024, 0, s>>>(hist, hist + bins);
+    xs::k_sort_scan_add<<<blocks, 1024, 0, s>>>(hist, hist + bins);
     xs::k_sort_scatter<<<grid_blocks(ctx, (int64_t)n, 256), 256, 0, s>>>(n, key, rec1, hist, rec0);
 #endif
     GTR_CUDA_TRY(cudaGetLastError());
