@@ -441,10 +441,19 @@ def run_gtr(a):
         flops = visits * FLOPS_PER_NUCLIDE
         achieved = flops / (k_ms * 1e-3) / 1e12
         traffic, traffic_src = ncu_traffic("r*_xs_sorted_ncu.json", "kernel_rt_sorted<Cfg<3, 3, 1, 256")
+        pipes = None           # hardware utilisation of the same kernel from the committed capture
+        profs = sorted(glob.glob(os.path.join(ROOT, "profiles", "r*_xs_sorted_ncu.json")))
+        if profs:
+            ks = [k for k in json.load(open(profs[-1]))["kernels"] if "kernel_rt_sorted<Cfg<3, 3, 1, 256" in k["kernel"]]
+            if ks:
+                pipes = {"fp64_pipe_active_pct": ks[0].get("sm__pipe_fp64_cycles_active.avg.pct_of_peak_sustained_active"),
+                         "issue_active_pct": ks[0].get("smsp__issue_active.avg.pct_of_peak_sustained_active"),
+                         "warp_instructions": ks[0].get("smsp__inst_executed.sum"),
+                         "source": os.path.relpath(profs[-1], ROOT)}
         roofline = {"bound": "alu", "achieved": achieved, "peak": fp64, "unit": "TFLOP/s",
                     "frac": achieved / fp64, "traffic": traffic, "traffic_source": traffic_src,
                     "kernel": "kernel_rt_sorted<SPMD, heap-to-stack, fold, 256> (the lookups in sorted order)",
-                    "kernel_ms": k_ms, "sort_ms": sort_ms, "alg_flops_per_launch": flops,
+                    "kernel_ms": k_ms, "sort_ms": sort_ms, "alg_flops_per_launch": flops, "ncu": pipes,
                     "peak_source": fp64_src,
                     "gather_model": {"alg_bytes_per_launch": alg_bytes, "unit": "GB/s",
                                      "achieved_kernel": alg_bytes / (k_ms * 1e-3) / 1e9,
