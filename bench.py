@@ -6,11 +6,15 @@ x 11,303 gridpoints, 17M lookups per GPU (weak scaling), synthetic seeded
 tables (gtr_inputs).  One step = one batch of 17M lookups through libgtr's
 headline variant (SPMD-ized + heap-to-stack + folding, thread_limit 256 --
 the paper's optimized form of XSBench's `target teams distribute parallel
-for`) plus, for N > 1, the combine of the 18 u64 hash/tallies: fused into
-the kernel's epilogue over peer memory (dist.PeerCombine), checked once
-against an NCCL all-reduce after warm-up (NCCL is used if they differ).
+for`) in XSBench's sorted event mode (sampling pass + sort by material and
+grid-index bucket + warp-coherent lookups, all inside the step; `--schedule
+bucketed` times the per-chunk bucketed schedule instead, which the line
+reports beside the headline either way) plus, for N > 1, the combine of the
+18 u64 hash/tallies: fused into the kernel's epilogue over peer memory
+(dist.PeerCombine), checked once against an NCCL all-reduce after warm-up
+(NCCL is used if they differ).
 
-    python bench.py [--gpus N] [--steps K] [--warmup W] [--impl gtr|reference]
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--impl gtr|reference] [--schedule sorted|bucketed]
     torchrun --nproc-per-node N bench.py --gpus N ...
 
 Rank 0 prints one JSON line.  `--impl reference` times the oracle (plain C on
